@@ -1,0 +1,358 @@
+"""Pins for the CPU oracle (oracle/): every check here is fixed by something
+other than the oracle itself — a closed form, an independent library routine
+(scipy.sparse.csgraph), a brute-force matrix-power BFS, a hand-computed value,
+or a number printed in the paper (tests/golden/).  CPU only."""
+import itertools
+import json
+import os
+
+import numpy as np
+import pytest
+import scipy.sparse as sp
+from scipy.sparse.csgraph import shortest_path
+
+import oracle
+
+GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
+
+
+def _graph(n, edges):
+    e = np.asarray(edges, dtype=np.int64).reshape(-1, 2)
+    return n, e[:, 0].astype(np.uint32), e[:, 1].astype(np.uint32)
+
+
+def _levels(n, edges, s):
+    n, src, dst = _graph(n, edges)
+    g = oracle.build_csr(n, src, dst)
+    level, parent, nl = oracle.bfs(g, s)
+    assert oracle.validate(g, src, dst, s, level, parent) == 0
+    return level, parent, nl
+
+
+# ---------------------------------------------------------------- closed forms
+
+def test_path_levels():
+    n = 37
+    for s in (0, 5, 36):
+        level, parent, nl = _levels(n, [(i, i + 1) for i in range(n - 1)], s)
+        assert np.array_equal(level, np.abs(np.arange(n) - s))
+        assert nl == max(s, n - 1 - s) + 1
+
+
+def test_cycle_levels():
+    n = 41
+    d = np.arange(n)
+    for s in (0, 17):
+        level, _, _ = _levels(n, [(i, (i + 1) % n) for i in range(n)], s)
+        assert np.array_equal(level, np.minimum(np.abs(d - s), n - np.abs(d - s)))
+
+
+def test_star_levels_and_parents():
+    n = 50
+    edges = [(0, i) for i in range(1, n)]
+    level, parent, _ = _levels(n, edges, 0)
+    assert level[0] == 0 and np.all(level[1:] == 1) and np.all(parent[1:] == 0)
+    level, parent, _ = _levels(n, edges, 7)          # from a leaf
+    expect = np.full(n, 2); expect[7] = 0; expect[0] = 1
+    assert np.array_equal(level, expect)
+    assert parent[0] == 7 and all(parent[v] == 0 for v in range(1, n) if v != 7)
+
+
+def test_complete_graph():
+    n = 16
+    level, _, nl = _levels(n, list(itertools.combinations(range(n), 2)), 3)
+    assert level[3] == 0 and np.all(np.delete(level, 3) == 1) and nl == 2
+
+
+def test_binary_tree():
+    n = 255
+    level, parent, _ = _levels(n, [((v - 1) // 2, v) for v in range(1, n)], 0)
+    assert np.array_equal(level, np.floor(np.log2(np.arange(n) + 1)).astype(int))
+    assert all(parent[v] == (v - 1) // 2 for v in range(1, n))
+
+
+def test_hypercube_popcount():
+    d = 8
+    n = 1 << d
+    edges = [(v, v ^ (1 << b)) for v in range(n) for b in range(d) if v < v ^ (1 << b)]
+    for s in (0, 0b10110011):
+        level, _, nl = _levels(n, edges, s)
+        assert np.array_equal(level, [bin(v ^ s).count("1") for v in range(n)])
+        assert nl == d + 1
+
+
+def test_grid_manhattan():
+    W, H = 23, 17
+    idx = lambda x, y: y * W + x
+    edges = [(idx(x, y), idx(x + 1, y)) for y in range(H) for x in range(W - 1)]
+    edges += [(idx(x, y), idx(x, y + 1)) for y in range(H - 1) for x in range(W)]
+    sx, sy = 5, 11
+    level, _, _ = _levels(W * H, edges, idx(sx, sy))
+    xs, ys = np.meshgrid(np.arange(W), np.arange(H))
+    assert np.array_equal(level, (np.abs(xs - sx) + np.abs(ys - sy)).ravel())
+
+
+def test_disjoint_union_unreached():
+    a = [(i, i + 1) for i in range(9)]           # 0..9 path
+    b = [(10 + i, 10 + i + 1) for i in range(4)]  # 10..14 path
+    level, parent, _ = _levels(20, a + b, 3)      # 15..19 isolated
+    assert np.all(level[10:] == -1) and np.all(parent[10:] == -1)
+    assert np.array_equal(level[:10], np.abs(np.arange(10) - 3))
+
+
+def test_isolated_source():
+    level, parent, nl = _levels(6, [(0, 1), (1, 2)], 5)
+    assert level[5] == 0 and parent[5] == 5 and nl == 1
+    assert np.all(np.delete(level, 5) == -1)
+
+
+def test_self_loops_and_multi_edges_have_no_effect():
+    base = [(i, i + 1) for i in range(11)]
+    noisy = base + [(3, 3), (7, 7), (2, 3), (3, 2), (2, 3), (0, 1)]
+    l1, _, _ = _levels(12, base, 0)
+    l2, _, _ = _levels(12, noisy, 0)
+    assert np.array_equal(l1, l2)
+    n, src, dst = _graph(12, noisy)
+    assert oracle.build_csr(n, src, dst).arcs == 22
+
+
+# ------------------------------------------------- brute force / library pins
+
+def _random_graph(rng, n, m):
+    e = rng.integers(0, n, size=(m, 2))
+    return e
+
+
+@pytest.mark.parametrize("seed", range(12))
+def test_bfs_matches_scipy_shortest_path(seed):
+    rng = np.random.default_rng(seed)
+    n = int(rng.integers(2, 64))
+    e = _random_graph(rng, n, int(rng.integers(0, 3 * n)))
+    n, src, dst = _graph(n, e)
+    g = oracle.build_csr(n, src, dst)
+    mask = src != dst
+    A = sp.coo_matrix((np.ones(mask.sum()), (src[mask], dst[mask])), shape=(n, n)).tocsr()
+    D = shortest_path(A, directed=False, unweighted=True)
+    for s in range(n):
+        level, parent, _ = oracle.bfs(g, s)
+        expect = np.where(np.isinf(D[s]), -1, D[s]).astype(np.int64)
+        assert np.array_equal(level, expect)
+        assert oracle.validate(g, src, dst, s, level, parent) == 0
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_bfs_matches_boolean_matrix_powers(seed):
+    """Textbook brute force: level k set = vertices first reached by A^k."""
+    rng = np.random.default_rng(100 + seed)
+    n = int(rng.integers(2, 60))
+    e = _random_graph(rng, n, int(rng.integers(n // 2, 2 * n + 1)))
+    n, src, dst = _graph(n, e)
+    adj = np.zeros((n, n), dtype=bool)
+    adj[src, dst] = True
+    adj[dst, src] = True
+    np.fill_diagonal(adj, False)
+    g = oracle.build_csr(n, src, dst)
+    for s in range(0, n, 3):
+        dist = np.full(n, -1)
+        reach = np.zeros(n, dtype=bool)
+        reach[s] = True
+        dist[s] = 0
+        k = 0
+        while True:
+            k += 1
+            nxt = (adj[reach].any(axis=0)) & ~reach & (dist == -1)
+            if not nxt.any():
+                break
+            dist[nxt] = k
+            reach = nxt
+        level, _, _ = oracle.bfs(g, s)
+        assert np.array_equal(level, dist)
+
+
+@pytest.mark.parametrize("seed", range(5))
+def test_csr_matches_set_build(seed):
+    rng = np.random.default_rng(200 + seed)
+    n = int(rng.integers(1, 1 << 12))
+    e = _random_graph(rng, n, int(rng.integers(0, 8 * n)))
+    n, src, dst = _graph(n, e)
+    g = oracle.build_csr(n, src, dst)
+    rows = [set() for _ in range(n)]
+    for u, v in zip(src.tolist(), dst.tolist()):
+        if u != v:
+            rows[u].add(v)
+            rows[v].add(u)
+    rp = np.concatenate([[0], np.cumsum([len(r) for r in rows])])
+    col = np.array([c for r in rows for c in sorted(r)], dtype=np.int32)
+    assert np.array_equal(g.row_ptr, rp)
+    assert np.array_equal(g.col, col)
+
+
+def test_reorder_invariants():
+    rng = np.random.default_rng(7)
+    n = 500
+    e = np.concatenate([rng.integers(0, n, (3000, 2)), np.stack([np.zeros(200, int), rng.integers(0, n, 200)], 1)])
+    n, src, dst = _graph(n, e)
+    g = oracle.build_csr(n, src, dst)
+    r = oracle.reorder(g)
+    deg = g.degree()
+    for v in range(n):
+        a, b = g.row_ptr[v], g.row_ptr[v + 1]
+        row = r.col[a:b]
+        assert sorted(row.tolist()) == g.col[a:b].tolist()                 # multiset preserved
+        keys = [(-int(deg[c]), int(c)) for c in row]
+        assert keys == sorted(keys)                                         # deg desc, id asc
+    # levels are invariant under the reorder (only parents change)
+    for s in (0, 13, 77):
+        assert np.array_equal(oracle.bfs(g, s)[0], oracle.bfs(r, s)[0])
+
+
+# ------------------------------------------------------------ validator pins
+
+def _valid_case():
+    rng = np.random.default_rng(11)
+    n = 200
+    e = rng.integers(0, n, (800, 2))
+    n, src, dst = _graph(n, e)
+    g = oracle.build_csr(n, src, dst)
+    s = int(src[0])
+    level, parent, _ = oracle.bfs(g, s)
+    return g, src, dst, s, level, parent
+
+
+def test_validator_accepts_oracle_tree():
+    g, src, dst, s, level, parent = _valid_case()
+    assert oracle.validate(g, src, dst, s, level, parent) == 0
+
+
+def test_validator_rejects_mutations():
+    g, src, dst, s, level, parent = _valid_case()
+    reached = np.flatnonzero((level >= 2))
+    v = int(reached[0])
+
+    p = parent.copy(); p[s] = int(reached[1])                        # wrong root parent
+    assert oracle.validate(g, src, dst, s, level, p) & oracle.V1_ROOT
+
+    # parent = a non-neighbour at the right level (tree edge missing)
+    same = [u for u in np.flatnonzero(level == level[v] - 1) if not
+            np.isin(v, g.col[g.row_ptr[u]:g.row_ptr[u + 1]])]
+    p = parent.copy(); p[v] = int(same[0])
+    assert oracle.validate(g, src, dst, s, level, p) & oracle.V4_TREE_EDGE
+
+    # parent at the same level (level step broken)
+    p = parent.copy(); p[v] = int(np.flatnonzero(level == level[v])[0 if np.flatnonzero(level == level[v])[0] != v else 1])
+    assert oracle.validate(g, src, dst, s, level, p) & (oracle.V3_LEVEL_STEP | oracle.V4_TREE_EDGE)
+
+    # 2-cycle between two reached vertices
+    u = int(parent[v]); p = parent.copy(); p[u] = v
+    assert oracle.validate(g, src, dst, s, level, p) != 0
+
+    # reached vertex marked unreached in level only
+    lv = level.copy(); lv[v] = -1
+    assert oracle.validate(g, src, dst, s, lv, parent) & oracle.V2_REACH
+
+    # level off by one everywhere at depth >= 2 (tree still consistent? no: V3/V5)
+    lv = level.copy(); lv[level >= 2] += 1
+    assert oracle.validate(g, src, dst, s, lv, parent) != 0
+
+    # an unreached vertex marked reached with a bogus parent
+    un = np.flatnonzero(level == -1)
+    if un.size:
+        lv = level.copy(); p = parent.copy(); lv[un[0]] = 1; p[un[0]] = s
+        assert oracle.validate(g, src, dst, s, lv, p) != 0
+
+
+# ----------------------------------------------------------- TEPS / stats pins
+
+def test_input_edges_grid_equals_m():
+    W, H = 9, 7
+    idx = lambda x, y: y * W + x
+    edges = [(idx(x, y), idx(x + 1, y)) for y in range(H) for x in range(W - 1)]
+    edges += [(idx(x, y), idx(x, y + 1)) for y in range(H - 1) for x in range(W)]
+    n, src, dst = _graph(W * H, edges)
+    g = oracle.build_csr(n, src, dst)
+    level, _, _ = oracle.bfs(g, 0)
+    assert oracle.input_edges(src, level) == 2 * W * H - W - H
+
+
+def test_input_edges_counts_duplicates_and_self_loops():
+    # component {0,1,2} + {3,4}; tuples with reached first endpoint from s=0
+    edges = [(0, 1), (1, 0), (0, 1), (2, 2), (1, 2), (3, 4), (4, 4)]
+    n, src, dst = _graph(5, edges)
+    g = oracle.build_csr(n, src, dst)
+    level, _, _ = oracle.bfs(g, 0)
+    assert oracle.input_edges(src, level) == 5
+
+
+def test_level_stats_star_hand_values():
+    n = 11
+    n, src, dst = _graph(n, [(0, i) for i in range(1, n)])
+    g = oracle.build_csr(n, src, dst)
+    level, _, _ = oracle.bfs(g, 0)
+    fs, fe = oracle.level_stats(g, level)
+    assert fs.tolist() == [1, 10] and fe.tolist() == [10, 10]
+
+
+def test_selector_paper_rule_on_table3():
+    """P:L87 + alpha = 0.1: on the Tab III ratios the rule selects BU
+    exactly at levels 3 and 4 — the levels where Tab VI's best is BU."""
+    gold = json.load(open(os.path.join(GOLDEN, "paper_r25.json")))
+    arcs = gold["rmat25_edges"]["value"]
+    ratios = gold["tab3_ratios"]["value"]
+    best = gold["tab6_best"]["value"]
+    picks = [oracle.select(1, 1, int(round(r * arcs)), arcs, alpha=gold["alpha"]["value"]) for r in ratios]
+    assert [p == 2 for p in picks] == [b == "BU" for b in best]
+    # strict '>' (reading C-8): ratio exactly alpha stays top-down
+    assert oracle.select(5, 1, 10, 100, alpha=0.1) != 2
+    assert oracle.select(5, 1, 11, 100, alpha=0.1) == 2
+    # growth rule (reading C-10): growing frontier -> SS, shrinking -> SF
+    assert oracle.select(100, 10, 50, 100000, alpha=0.1, grow=2.0, ratio_min=1e-4) == 1
+    assert oracle.select(10, 100, 50, 100000, alpha=0.1, grow=2.0, ratio_min=1e-4) == 0
+
+
+def test_byte_replay_hand_computed():
+    """Path 0-1-2-3 from s=0 (n=4, A=6); strategies SF, BU, SF.
+    deg = [1,2,2,1]; F = {0},{1},{2},{3}.
+      init         8*4 + 4*ceil(4/8)=4                     = 36
+      L0 SF        20*1 + 4*1 + 28*1                       = 52
+      L1 BU        n/4=1 + n/8=0 + 16*U_1(=2: {2,3}) + 4*probes + 8*1
+                   probes: v2 row [1,3] (reordered by deg desc: 1 (deg 2) then 3) -> 1
+                           v3 row [2] -> no level-1 neighbour -> deg = 1   => 2
+                   = 1 + 0 + 32 + 8 + 8                     = 49
+      L2 SF        after BU: generate n/8=0 + 28*1; 20*1 + 4*2 + 28*1 = 84
+      L3 SF        20*1 + 4*1 + 0                           = 24
+    """
+    n, src, dst = _graph(4, [(0, 1), (1, 2), (2, 3)])
+    g = oracle.reorder(oracle.build_csr(n, src, dst))
+    level, _, nl = oracle.bfs(g, 0)
+    assert nl == 4
+    tot, per = oracle.byte_replay(g, level, [0, 2, 0, 0])
+    assert per.tolist() == [52, 49, 84, 24]
+    assert tot == 36 + 52 + 49 + 84 + 24
+
+
+# ------------------------------------------------------- paper byte model pin
+
+def test_paper_bandwidth_model_reproduces_13_7_percent():
+    from paper_conf_sc_yangls0w24_b200 import metrics
+    gold = json.load(open(os.path.join(GOLDEN, "paper_r25.json")))
+    V, M = gold["rmat25_vertices"]["value"], gold["rmat25_edges"]["value"]
+    b = metrics.model_bytes(V, M)
+    assert b == 2_684_335_432
+    # 43 GTEPS over |M| arcs gives the runtime; both efficiencies follow.
+    t = M / (gold["gteps"]["value"] * 1e9)
+    bw = gold["bandwidth_tbs"]["value"] * 1e12
+    assert abs(metrics.bandwidth_efficiency(b, t, bw) - gold["predicted_efficiency"]["value"]) < 0.005
+    hw = gold["hardware_bytes_gb"]["value"] * 1e9
+    assert abs(metrics.bandwidth_efficiency(hw, t, bw) - gold["hardware_efficiency"]["value"]) < 0.005
+    # Tab I "Sum" = levels 0..5 (reading C-21)
+    kb = gold["tab1_fetch_kb_rearranged"]["value"]
+    assert abs(sum(kb[:6]) - gold["tab1_sum_kb_rearranged"]["value"]) < 0.02
+    # Tab III ratios sum to ~1: every arc of the root's component expanded once
+    assert abs(sum(gold["tab3_ratios"]["value"]) - 0.999855) < 1e-5
+
+
+def test_harmonic_mean_and_quartiles():
+    from paper_conf_sc_yangls0w24_b200 import metrics
+    assert metrics.harmonic_mean([1.0, 2.0, 4.0]) == pytest.approx(3 / (1 + 0.5 + 0.25))
+    q = metrics.quartiles([1, 2, 3, 4, 5])
+    assert (q["min"], q["q1"], q["median"], q["q3"], q["max"]) == (1, 2, 3, 4, 5)
