@@ -1,0 +1,422 @@
+#!/usr/bin/env python
+"""XBFS on B200 — headline benchmark (BASELINE.json metric).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config s24] [--impl ours|reference]
+
+Metric: GTEPS per B200 on a Graph500 Kronecker graph (edgefactor 16), Graph500
+convention (m = input tuples of the reached component, O-6), harmonic mean over
+the timed roots.  A "step" is one complete BFS (init + every level) from one
+root; W untimed warm-up roots precede K timed roots.  Every timed BFS is
+preceded by an L2 flush (512 MiB write, outside the timed region).  Device
+time per BFS = CUDA events on the library stream around init .. last level.
+
+At N > 1 (torchrun, one process per GPU) every rank holds the same graph and
+runs its own K roots (independent problems: weak scaling, no data-path
+collective); value = N x min over ranks of the per-rank harmonic mean.
+
+--impl reference times the CPU oracle (oracle/, serial FIFO BFS, 1 thread) on
+the same graph and roots: the reference arm of this paper-only tier.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+if ROOT not in sys.path:
+    sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+METRIC = "GTEPS per B200 (Graph500 Kronecker, harmonic mean over 64 roots) at 1/2/4/8 GPU"
+
+CONFIGS = {
+    "s10": dict(kind="kron", scale=10, edgefactor=16),
+    "s16": dict(kind="kron", scale=16, edgefactor=16),
+    "s20": dict(kind="kron", scale=20, edgefactor=16),
+    "s22": dict(kind="kron", scale=22, edgefactor=16),
+    "s24": dict(kind="kron", scale=24, edgefactor=16),
+    "s25": dict(kind="kron", scale=25, edgefactor=16),
+    "grid": dict(kind="grid", width=4096, height=4096),
+}
+GRAPH_SEED, ROOT_SEED = 1, 2
+
+
+def workload_name(cfg_name: str) -> str:
+    c = CONFIGS[cfg_name]
+    if c["kind"] == "kron":
+        return f"graph500-kronecker-s{c['scale']}-ef{c['edgefactor']}"
+    return f"grid-{c['width']}x{c['height']}"
+
+
+def make_graph(cfg_name: str, pinned: bool):
+    from paper_conf_sc_yangls0w24_b200 import synth
+    c = CONFIGS[cfg_name]
+    if c["kind"] == "kron":
+        return synth.kronecker(c["scale"], c["edgefactor"], seed=GRAPH_SEED, pinned=pinned)
+    src, dst, n = synth.grid(c["width"], c["height"], seed=GRAPH_SEED)
+    return src, dst, n
+
+
+def pick_roots(cfg_name: str, n, src, dst, count: int):
+    from paper_conf_sc_yangls0w24_b200 import synth
+    c = CONFIGS[cfg_name]
+    if c["kind"] == "grid":
+        W, H = c["width"], c["height"]
+        fixed = [0, (H // 2) * W + W // 2]
+        rnd = synth.roots(n, src, dst, count + 2, root_seed=ROOT_SEED).tolist()
+        out = fixed + [r for r in rnd if r not in fixed]
+        return np.array(out[:count], dtype=np.int64)
+    return synth.roots(n, src, dst, count, root_seed=ROOT_SEED)
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    except Exception:
+        return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+
+    FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+              "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device: int):
+        self.device = device
+        self.proc = None
+        self.lines = []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.device), f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
+                 "-lms", "100"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self._t = threading.Thread(target=self._read, daemon=True)
+            self._t.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if not self.proc:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        time.sleep(0.25)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            parts = [p.strip() for p in ln.split(",")]
+            if len(parts) < 7:
+                continue
+            try:
+                sm.append(float(parts[0]))
+                mx.append(float(parts[1]))
+            except ValueError:
+                continue
+            for nm, val in zip(names, parts[3:7]):
+                if val.lower().startswith("active"):
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def kernel_bytes(name: str, level: int, st, n: int) -> int:
+    """Algorithmic bytes of one launch, from the run's per-level counters."""
+    from paper_conf_sc_yangls0w24_b200 import metrics
+    if name == "init_fill":
+        return metrics.bytes_init(n)
+    if level < 0 or level >= st.num_levels:
+        return 0
+    fv, fe = st.frontier_vertices[level], st.frontier_edges[level]
+    found = st.frontier_vertices[level + 1] if level + 1 < st.num_levels else 0
+    if name == "td_expand_sf":
+        return metrics.bytes_td_sf(n, fv, fe, found)
+    if name == "td_expand_ss":
+        return metrics.bytes_td_ss(n, fv, fe, found)
+    if name == "generate_pre":
+        return metrics.bytes_generate(n, fv, post=False)
+    if name == "generate_post":
+        return metrics.bytes_generate(n, found, post=True)
+    if name == "bu_traverse":
+        return metrics.bytes_bu(n, st.unvisited[level], st.bu_probes[level], found)
+    return 0
+
+
+def run_ours(args):
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_sc_yangls0w24_b200 import metrics
+    from paper_conf_sc_yangls0w24_b200.xbfs import Graph
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device(f"cuda:{local}"))
+    torch.cuda.set_device(local)
+    dev = torch.device(f"cuda:{local}")
+    t0 = time.time()
+    src, dst, n = make_graph(args.config, pinned=True)
+    t_gen = time.time() - t0
+    total_roots = args.warmup + args.steps * world
+    roots = pick_roots(args.config, n, src, dst, total_roots)
+    if len(roots) < total_roots:
+        roots = np.resize(roots, total_roots)
+    warm = roots[: args.warmup]
+    mine = roots[args.warmup + rank * args.steps: args.warmup + (rank + 1) * args.steps]
+
+    stream = torch.cuda.current_stream(dev)
+    t0 = time.time()
+    g = Graph(torch.from_numpy(src.view(np.int32)), torch.from_numpy(dst.view(np.int32)), n, device=local,
+              stream=stream.cuda_stream, reorder=False)
+    torch.cuda.synchronize()
+    t_build = time.time() - t0
+    t0 = time.time()
+    g.reorder(1)
+    torch.cuda.synchronize()
+    t_reorder = time.time() - t0
+    level = torch.empty(n, dtype=torch.int32, device=dev)
+    parent = torch.empty(n, dtype=torch.int32, device=dev)
+    flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
+    opts = dict(driver=args.driver)
+
+    for r in warm:
+        g.run(int(r), level, parent, stats=True, **opts)
+    torch.cuda.synchronize()
+
+    clocks = ClockSampler(local)
+    clocks.start()
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    per_root = []
+    launches = 0
+    for r in mine:
+        flush.fill_(1)                       # L2 flush, outside the timed region
+        _, _, st = g.run(int(r), level, parent, stats=True, **opts)
+        per_root.append((int(r), st.elapsed_ms, st.input_edges_traversed, st.arcs_traversed, st.num_levels,
+                         "".join("FSB"[s] for s in st.strategy)))
+        launches += st.kernel_launches
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    clk = clocks.stop()
+
+    teps = [m / (ms * 1e-3) for (_, ms, m, _, _, _) in per_root]
+    teps_arcs = [a / (ms * 1e-3) for (_, ms, _, a, _, _) in per_root]
+    hmean = metrics.harmonic_mean(teps)
+    ms_mean = statistics.mean(ms for (_, ms, *_rest) in per_root)
+
+    # parity spot check of the last timed root against a fresh run's invariants is in tests;
+    # here: the parent tree of the last timed root must be consistent (cheap device check)
+    lv = level.cpu().numpy()
+    pa = parent.cpu().numpy()
+    r_last = per_root[-1][0]
+    ok_root = lv[r_last] == 0 and pa[r_last] == r_last
+    reached = lv >= 0
+    ok_tree = bool(ok_root and np.all(lv[pa[reached & (np.arange(n) != r_last)]] ==
+                                      lv[reached & (np.arange(n) != r_last)] - 1))
+
+    # e2e: public C-ABI call with HOST output buffers (D2H of level+parent inside)
+    lh = torch.empty(n, dtype=torch.int32, pin_memory=True).numpy()
+    ph = torch.empty(n, dtype=torch.int32, pin_memory=True).numpy()
+    e2e_t = []
+    for r in mine[: min(len(mine), args.e2e_roots)]:
+        flush.fill_(1)
+        torch.cuda.synchronize()
+        t1 = time.perf_counter()
+        g.run_host(int(r), lh, ph, **opts)
+        e2e_t.append(time.perf_counter() - t1)
+    m_of = {r: m for (r, _, m, *_rest) in per_root}
+    e2e_teps = [m_of[int(r)] / t for r, t in zip(mine, e2e_t)]
+
+    # roofline: per-launch event timing of a few roots (host-loop driver)
+    peak, peak_src = load_peaks()
+    agg = {}
+    for r in mine[: min(len(mine), args.profile_roots)]:
+        flush.fill_(1)
+        _, _, st = g.run(int(r), level, parent, stats=True, profile=8192, driver=1)
+        for (name, lvl, ms) in st.kernels:
+            b = kernel_bytes(name, lvl, st, n)
+            a = agg.setdefault(name, [0, 0.0, 0])
+            a[0] += 1
+            a[1] += ms
+            a[2] += b
+    kernels = {k: {"launches": v[0], "total_ms": round(v[1], 4), "avg_ms": round(v[1] / v[0], 5),
+                   "bytes_per_launch": int(v[2] / v[0]),
+                   "gbs": round(v[2] / (v[1] * 1e-3) / 1e9, 1) if v[1] > 0 else None}
+               for k, v in agg.items()}
+    dom = max(agg.items(), key=lambda kv: kv[1][1])[0] if agg else None
+    roofline = None
+    if dom:
+        d = kernels[dom]
+        ach = d["gbs"]
+        roofline = {"bound": "hbm", "kernel": dom, "achieved": ach, "peak": peak, "unit": "GB/s",
+                    "frac": round(ach / peak, 4) if ach else None, "traffic": None,
+                    "bytes_per_launch": d["bytes_per_launch"], "peak_source": peak_src}
+    b_model = metrics.model_bytes(n, g.arcs)
+    model_frac = b_model / (ms_mean * 1e-3) / (peak * 1e9)
+
+    res = dict(rank=rank, hmean=hmean, per_root=per_root, launches=launches, ms_mean=ms_mean,
+               e2e=metrics.harmonic_mean(e2e_teps) if e2e_teps else None, clocks=clk, ok_tree=ok_tree,
+               roofline=roofline, kernels=kernels, teps_arcs=metrics.harmonic_mean(teps_arcs),
+               model_frac=model_frac, quart=metrics.quartiles(teps))
+    if world > 1:
+        allres = [None] * world
+        dist.all_gather_object(allres, res)
+    else:
+        allres = [res]
+    if rank != 0:
+        g.close()
+        if world > 1:
+            dist.destroy_process_group()
+        return
+
+    worst = min(allres, key=lambda x: x["hmean"])
+    value = world * worst["hmean"] / 1e9
+    cpu = None
+    if world == 1 and not args.no_cpu_baseline:
+        cpu = cpu_baseline(args, src, dst, n, mine, m_of)
+    line = {
+        "metric": METRIC,
+        "value": round(value, 3),
+        "unit": "GTEPS",
+        "n_gpus": world,
+        "steps": args.steps,
+        "warmup": args.warmup,
+        "ms_per_step": round(max(x["ms_mean"] for x in allres), 4),
+        "higher_is_better": True,
+        "scaling": "weak",
+        "vs_baseline": None,
+        "dtype": "int32",
+        "data": "synthetic (seeded Graph500 Kronecker generator, graph seed 1, root seed 2)",
+        "config": {"workload": workload_name(args.config), "n_vertices": n, "input_edges": int(src.shape[0]),
+                   "arcs": g.arcs, "roots_per_gpu": args.steps, "l2_flush": "512 MiB write before every timed BFS",
+                   "reorder": "degree-desc (P:L153)", "alpha": 0.1, "driver": args.driver,
+                   "parallelism": f"replicas x{world} (independent roots)"},
+        "gteps_hmean_per_gpu": round(worst["hmean"] / 1e9, 3),
+        "gteps_arcs_hmean": round(res["teps_arcs"] / 1e9, 3),
+        "gteps_quartiles": {k: round(v / 1e9, 3) for k, v in res["quart"].items()},
+        "roofline_model": {"bytes": b_model, "formula": "16N + 4A (P:L358)", "frac": round(model_frac, 4),
+                           "peak_gbs": peak},
+        "clocks": res["clocks"],
+        "e2e": {"value": round(res["e2e"] / 1e9, 3) if res["e2e"] else None, "unit": "GTEPS",
+                "h2d_bytes_per_step": 8, "d2h_bytes_per_step": 8 * n,
+                "note": "xbfs_run_host: source scalar in, level+parent (int32 each) D2H into pinned memory"},
+        "gpu_launches": int(sum(x["launches"] for x in allres)),
+        "roofline": res["roofline"],
+        "kernels": res["kernels"],
+        "cpu_baseline": cpu,
+        "levels": [pr[4] for pr in res["per_root"][:4]],
+        "strategies": [pr[5] for pr in res["per_root"][:4]],
+        "parent_tree_consistent": bool(all(x["ok_tree"] for x in allres)),
+        "prep_s": {"generate": round(t_gen, 2), "build_csr": round(t_build, 2), "reorder": round(t_reorder, 2)},
+    }
+    print(json.dumps(line), flush=True)
+    g.close()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def cpu_baseline(args, src, dst, n, roots, m_of=None, budget_s=None):
+    """The oracle as it stands (serial FIFO BFS, 1 thread) on a bounded sample of
+    the same workload: the first roots until ~budget seconds of BFS time."""
+    import oracle
+    budget_s = args.cpu_budget if budget_s is None else budget_s
+    t0 = time.time()
+    og = oracle.build_csr(n, src, dst)
+    t_csr = time.time() - t0
+    teps, used, spent = [], [], 0.0
+    for r in roots:
+        t1 = time.perf_counter()
+        lv, _, _ = oracle.bfs(og, int(r))
+        dt = time.perf_counter() - t1
+        m = oracle.input_edges(src, lv)
+        teps.append(m / dt)
+        used.append(int(r))
+        spent += dt
+        if spent >= budget_s:
+            break
+    from paper_conf_sc_yangls0w24_b200 import metrics
+    return {"value": round(metrics.harmonic_mean(teps) / 1e9, 5), "unit": "GTEPS", "cores": 1, "kind": "oracle",
+            "sample": f"{len(used)} of the timed roots of {workload_name(args.config)} (serial BFS, oracle CSR "
+                      f"prebuilt in {t_csr:.1f}s untimed), {spent:.1f}s of BFS",
+            "host_cores": os.cpu_count()}
+
+
+def run_reference(args):
+    """Reference arm: the CPU oracle timed as it stands (rank 0 only)."""
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    import oracle
+    from paper_conf_sc_yangls0w24_b200 import metrics
+    src, dst, n = make_graph(args.config, pinned=False)
+    roots = pick_roots(args.config, n, src, dst, args.warmup + args.steps * world)
+    og = oracle.build_csr(n, src, dst)
+    for r in roots[: args.warmup]:
+        oracle.bfs(og, int(r))
+    teps, times = [], []
+    for r in roots[args.warmup: args.warmup + args.steps]:
+        t1 = time.perf_counter()
+        lv, _, _ = oracle.bfs(og, int(r))
+        dt = time.perf_counter() - t1
+        teps.append(oracle.input_edges(src, lv) / dt)
+        times.append(dt)
+    value = metrics.harmonic_mean(teps) / 1e9
+    line = {
+        "impl": "reference", "metric": METRIC, "value": round(value, 5), "unit": "GTEPS", "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(1e3 * statistics.mean(times), 3),
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
+        "config": {"workload": workload_name(args.config), "n_vertices": n, "input_edges": int(src.shape[0]),
+                   "arcs": og.arcs},
+        "cpu_baseline": {"value": round(value, 5), "unit": "GTEPS", "cores": 1, "kind": "oracle",
+                         "sample": f"{args.steps} roots, one full serial BFS each (oracle CSR prebuilt, untimed)"},
+        "e2e": {"value": round(value, 5), "unit": "GTEPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=64)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default="s24", choices=sorted(CONFIGS))
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--driver", type=int, default=0, help="0 auto, 1 host loop, 2 CUDA-graph device loop")
+    ap.add_argument("--e2e-roots", type=int, default=8)
+    ap.add_argument("--profile-roots", type=int, default=4)
+    ap.add_argument("--cpu-budget", type=float, default=15.0)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args()
+    assert args.warmup >= 3 or args.impl == "reference" or os.environ.get("XBFS_ALLOW_SHORT_WARMUP"), \
+        "timing rules: at least 3 warm-up steps"
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_ours(args)
+
+
+if __name__ == "__main__":
+    main()

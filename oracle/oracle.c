@@ -212,21 +212,25 @@ int32_t oracle_select(int64_t f_size, int64_t f_prev, int64_t f_edges, int64_t a
 }
 
 /* ------------------------------------------------------ O-8 byte replay */
-/* Algorithmic bytes of one BFS (DESIGN.md §5 "B_alg"), given the strategy used
- * at each level (0 SF, 1 SS, 2 BU) and the (reordered) CSR the GPU traversed.
- *   init          : 8n (level+parent) + 4 * n/8 (visited + 3 frontier bitmaps)
- *   TD step k     : 20|F_k| (queue entry) + 4 edgesF_k (col) + 28 per vertex
- *                   discovered (level 4, parent 4, row_ptr 16, queue 4... see
- *                   DESIGN.md) ; SS adds n/8 (bitmap generation scan)
- *   BU step k     : n/4 (visited + nonisolated words) + n/8 (next words) +
- *                   16|U_k| (row_ptr pair) + 4*sum(probes) + 8*found
- *   generate      : n/8 + 28|F| when a TD step follows a BU step
+/* Algorithmic bytes of one BFS (the per-kernel model of DESIGN.md §5), given
+ * the strategy used at each level (0 SF, 1 SS, 2 BU) and the (reordered) CSR
+ * the GPU traversed.  B = 4*ceil(n/32) is one n-bit bitmap pass.
+ *   init        : 8n (level+parent) + 5B (visited, non-isolated, 3 frontier maps)
+ *   SF step k   : B (stale frontier clear) + 20|F_k| (queue entries) + 4 edgesF_k
+ *                 (col) + 44|F_{k+1}| (level 4, parent 4, row_ptr pair 16, queue 20)
+ *   SS step k   : B + 20|F_k| + 4 edgesF_k + 8|F_{k+1}|, then the generation scan
+ *                 2B + 36|F_{k+1}| (bitmap read, visited OR, row_ptr pair + queue)
+ *   BU step k   : 4B (visited read+write, next write, stale clear) + 16|U_k|
+ *                 (row_ptr pair per candidate) + 4 probes_k (col) + 8|F_{k+1}|
+ *   a TD step right after a BU step first rebuilds the queue: B + 36|F_k|.
  * probes(v) = 1 + index of the first level-k neighbour in v's stored row, or
- * deg(v) if none.  Also returns the per-level pieces in out[] (cap entries). */
+ * deg(v) if none (BU tests only level k: reading C-9).  per_level[k] gets the
+ * bytes of step k; the return value includes init. */
 int64_t oracle_byte_replay(int64_t n, const int64_t* row_ptr, const int32_t* col,
                            const int32_t* level, int32_t nlevels, const int8_t* strategy,
                            int64_t* per_level) {
-    int64_t total = 8 * n + 4 * ((n + 7) / 8);
+    const int64_t B = 4 * ((n + 31) / 32);
+    int64_t total = 8 * n + 5 * B;
     int64_t* fsize = (int64_t*)calloc((size_t)nlevels + 1, sizeof(int64_t));
     int64_t* fedges = (int64_t*)calloc((size_t)nlevels + 1, sizeof(int64_t));
     if (!fsize || !fedges) { free(fsize); free(fedges); return -1; }
@@ -253,12 +257,13 @@ int64_t oracle_byte_replay(int64_t n, const int64_t* row_ptr, const int32_t* col
                     if (level[col[p]] == k) { pr = p - row_ptr[v] + 1; break; }
                 probes += pr;
             }
-            bytes = n / 4 + n / 8 + 16 * unvisited + 4 * probes + 8 * found;
+            bytes = 4 * B + 16 * unvisited + 4 * probes + 8 * found;
             prev_bu = 1;
         } else {
-            if (prev_bu) bytes += n / 8 + 28 * fsize[k];        /* queue generation */
-            bytes += 20 * fsize[k] + 4 * fedges[k] + 28 * found;
-            if (strategy[k] == 1) bytes += n / 8;               /* single-scan pass */
+            if (prev_bu) bytes += B + 36 * fsize[k];            /* queue rebuilt from the bitmap */
+            bytes += B + 20 * fsize[k] + 4 * fedges[k];
+            if (strategy[k] == 0) bytes += 44 * found;
+            else bytes += 8 * found + 2 * B + 36 * found;       /* single-scan generation */
             prev_bu = 0;
         }
         unvisited -= found;

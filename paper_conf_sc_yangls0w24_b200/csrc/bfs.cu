@@ -1,0 +1,650 @@
+// bfs.cu — the XBFS level kernels for sm_100a and the level-loop drivers.
+//
+// Per level k (§III):
+//   SF  td_expand<SF>: atomic test-and-set on the visited bitmap;
+//                    the winner writes level/parent and is appended to the next
+//                    queue with ONE packed 64-bit atomic per warp that returns
+//                    both its slot and its degree offset (edge-balanced tiles).
+//   SS [generate if the queue is missing] + td_expand<SS> (plain
+//                    level/parent stores, no status atomics; next-frontier bit
+//                    set with a fire-and-forget RED) + generate (one scan of the
+//                    next-frontier bitmap builds the next queue).  When a queue
+//                    already exists (after SF/SS) the first generate is skipped:
+//                    No-Frontier-Generation.
+//   BU bu_traverse: each warp takes 32 bitmap words (1024
+//                    vertices), compacts the unvisited ones with ballot/popc
+//                    (the paper's count + prefix-sum + queue-write "double scan"
+//                    folded into registers and shared memory), then each lane
+//                    walks one candidate's (degree-ordered) row and stops
+//                    at the first neighbour in the current frontier bitmap.
+//   select (1 thread): consolidates the counters, logs the level, and picks the
+//                    next strategy: BU iff edgesF/A > alpha, else
+//                    SS/SF by frontier growth (reading C-10).
+#include <stdio.h>
+#include <string.h>
+
+#include <algorithm>
+
+#include "common.cuh"
+
+namespace xbfs {
+
+constexpr unsigned FULL = 0xffffffffu;
+
+__device__ __forceinline__ void count_launch(DevState* st) {
+    if (blockIdx.x == 0 && threadIdx.x == 0) atomicAdd(&st->launches, 1u);
+}
+
+// Clear the stale frontier bitmap fb[(k+2)%3] (it held F_{k-1}); it becomes the
+// "next" bitmap of level k+1.  Grid-stride, vectorised.
+__device__ __forceinline__ void clear_stale(const KArgs& a, int k) {
+    unsigned int* z = a.fb[(k + 2) % 3];
+    const long long w4 = a.words / 4;
+    uint4* z4 = reinterpret_cast<uint4*>(z);
+    const long long tid = blockIdx.x * (long long)blockDim.x + threadIdx.x;
+    const long long nth = (long long)gridDim.x * blockDim.x;
+    for (long long i = tid; i < w4; i += nth) z4[i] = make_uint4(0, 0, 0, 0);
+    for (long long i = w4 * 4 + tid; i < a.words; i += nth) z[i] = 0;
+}
+
+// Warp-aggregated enqueue of the lanes with `win` set: one 64-bit atomicAdd on
+// the packed counter returns both the queue slot base (high bits) and the degree
+// offset base (low dbits), so qoff is an exact exclusive prefix sum of degrees
+// over the queue, in slot order.  Every tile start (multiple of kTile) that falls
+// inside a vertex's arc range records that vertex's slot in tile_first.
+__device__ __forceinline__ void enqueue_warp(bool win, int v, long long rs, long long deg,
+                                             unsigned long long* ctr, int dbits, int* qv, long long* qoff,
+                                             long long* qdelta, int* tile_first) {
+    const unsigned mask = __ballot_sync(FULL, win);
+    if (mask == 0) return;
+    const int lane = threadIdx.x & 31;
+    const int rank = __popc(mask & ((1u << lane) - 1u));
+    long long d = win ? deg : 0;
+    long long incl = d;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        long long t = __shfl_up_sync(FULL, incl, o);
+        if (lane >= o) incl += t;
+    }
+    const long long total = __shfl_sync(FULL, incl, 31);
+    unsigned long long base = 0;
+    if (lane == 0)
+        base = atomicAdd(ctr, ((unsigned long long)__popc(mask) << dbits) + (unsigned long long)total);
+    base = __shfl_sync(FULL, base, 0);
+    if (win) {
+        const long long slot = (long long)(base >> dbits) + rank;
+        const long long off = (long long)(base & ((1ull << dbits) - 1ull)) + incl - d;
+        qv[slot] = v;
+        qoff[slot] = off;
+        qdelta[slot] = rs - off;
+        if (deg > 0) {
+            const long long t0 = (off + kTile - 1) / kTile, t1 = (off + deg - 1) / kTile;
+            for (long long t = t0; t <= t1; ++t) tile_first[t] = (int)slot;
+        }
+    }
+}
+
+// ---------------------------------------------------------------- init
+__global__ __launch_bounds__(256) void k_init_fill(KArgs a, int* __restrict__ level, int* __restrict__ parent,
+                                                   const unsigned int* __restrict__ nonisolated) {
+    count_launch(a.st);
+    const long long tid = blockIdx.x * (long long)blockDim.x + threadIdx.x;
+    const long long nth = (long long)gridDim.x * blockDim.x;
+    const long long n4 = a.n / 4;
+    int4* l4 = reinterpret_cast<int4*>(level);
+    int4* p4 = reinterpret_cast<int4*>(parent);
+    const int4 m1 = make_int4(-1, -1, -1, -1);
+    if ((((uintptr_t)level | (uintptr_t)parent) & 15) == 0) {
+        for (long long i = tid; i < n4; i += nth) { l4[i] = m1; p4[i] = m1; }
+        for (long long i = n4 * 4 + tid; i < a.n; i += nth) { level[i] = -1; parent[i] = -1; }
+    } else {
+        for (long long i = tid; i < a.n; i += nth) { level[i] = -1; parent[i] = -1; }
+    }
+    // isolated vertices are pre-marked visited: never BU candidates (reading C-27)
+    for (long long w = tid; w < a.words; w += nth) {
+        a.visited[w] = ~nonisolated[w];
+        a.fb[0][w] = 0;
+        a.fb[1][w] = 0;
+        a.fb[2][w] = 0;
+    }
+}
+
+__device__ int choose_strategy(const DevState* st, long long arcs, long long fsize, long long fprev,
+                               long long fedges, long long unvisited, int prev) {
+    if (st->force >= 0) return st->force;
+    const double ratio = arcs > 0 ? (double)fedges / (double)arcs : 0.0;
+    if (ratio > st->alpha) return XBFS_BU;                                    // P:L87, strict (C-8)
+    if (st->bu_stay > 0.0 && prev == XBFS_BU && (double)unvisited * st->bu_stay < (double)fedges)
+        return XBFS_BU;                                                       // C-11 (optional)
+    if ((double)fsize > st->grow * (double)fprev && ratio > st->ratio_min) return XBFS_SS;  // C-10
+    return XBFS_SF;
+}
+
+// Seed the source (the source holds level 0) and reset the level state.
+__global__ void k_seed(KArgs a, int* level, int* parent, long long s, long long nonisolated_count) {
+    count_launch(a.st);
+    DevState* st = a.st;
+    const long long rs = a.row_ptr[s], deg = a.row_ptr[s + 1] - rs;
+    level[s] = 0;
+    parent[s] = (int)s;
+    a.visited[s >> 5] |= 1u << (s & 31);
+    a.fb[0][s >> 5] |= 1u << (s & 31);
+    a.qv[0][0] = (int)s;
+    a.qoff[0][0] = 0;
+    a.qdelta[0][0] = rs;
+    if (deg > 0) {
+        const long long t1 = (deg - 1) / kTile;
+        for (long long t = 0; t <= t1; ++t) a.tile_first[0][t] = 0;
+    }
+    st->k = 0;
+    st->qctr[0] = (1ull << a.dbits) + (unsigned long long)deg;
+    st->qctr[1] = 0;
+    st->queue_valid = 1;
+    st->done = 0;
+    st->fsize = 1;
+    st->fedges = deg;
+    st->fprev = 0;
+    st->unvisited = nonisolated_count - (deg > 0 ? 1 : 0);
+    st->acc_found = st->acc_edges = st->acc_probes = 0;
+    st->reached = 0;
+    st->arcs_traversed = 0;
+    st->nlevels = 0;
+    st->source = s;
+    st->prev_strategy = -1;
+    st->strategy = choose_strategy(st, a.arcs, 1, 0, deg, st->unvisited, -1);
+    a.hctl->k = 0;
+    a.hctl->strategy = st->strategy;
+    a.hctl->queue_valid = 1;
+    a.hctl->done = 0;
+}
+
+// ----------------------------------------------------------- top-down
+// One tile = kTile consecutive frontier arcs; tile_first gives the first queue
+// entry overlapping it, so tiles are balanced regardless of the degree mix
+// (hubs span many tiles, small vertices share one).  Arc a of the frontier is
+// col[a + qdelta[j]] for its owner j (binary search of qoff in shared memory).
+template <int MODE>
+__global__ __launch_bounds__(kExpandThreads, 4) void k_td_expand(KArgs a, int* __restrict__ level,
+                                                                int* __restrict__ parent) {
+    count_launch(a.st);
+    const int k = a.st->k;
+    clear_stale(a, k);
+    const int in = k & 1, ob = (k + 1) & 1;
+    const unsigned long long q = a.st->qctr[in];
+    const long long F = (long long)(q >> a.dbits);
+    const long long T = (long long)(q & ((1ull << a.dbits) - 1ull));
+    if (F == 0 || T == 0) return;
+    const long long ntiles = (T + kTile - 1) / kTile;
+    const int* __restrict__ qv = a.qv[in];
+    const long long* __restrict__ qoff = a.qoff[in];
+    const long long* __restrict__ qdelta = a.qdelta[in];
+    const int* __restrict__ tfirst = a.tile_first[in];
+    unsigned int* __restrict__ visited = a.visited;
+    unsigned int* __restrict__ next = a.fb[(k + 1) % 3];
+    const int lvl = k + 1;
+
+    __shared__ long long s_off[kTile + 1];
+    __shared__ long long s_delta[kTile + 1];
+    __shared__ int s_v[kTile + 1];
+
+    for (long long t = blockIdx.x; t < ntiles; t += gridDim.x) {
+        const long long a0 = t * kTile;
+        const long long a1 = min(a0 + (long long)kTile, T);
+        const long long i0 = tfirst[t];
+        const long long i1 = (t + 1 < ntiles) ? (long long)tfirst[t + 1] : F - 1;
+        const int nv = (int)(i1 - i0 + 1);
+        __syncthreads();
+        for (int i = threadIdx.x; i < nv; i += blockDim.x) {
+            s_off[i] = qoff[i0 + i];
+            s_delta[i] = qdelta[i0 + i];
+            s_v[i] = qv[i0 + i];
+        }
+        __syncthreads();
+        int j = 0;
+#pragma unroll 1
+        for (int it = 0; it < kTile / kExpandThreads; ++it) {
+            const long long arc = a0 + it * kExpandThreads + threadIdx.x;
+            const bool valid = arc < a1;
+            bool win = false;
+            int v = 0;
+            long long rs = 0, deg = 0;
+            if (valid) {
+                // owner: last j with s_off[j] <= arc (arcs of a thread increase)
+                int lo = j, hi = nv - 1;
+                while (lo < hi) {
+                    const int mid = (lo + hi + 1) >> 1;
+                    if (s_off[mid] <= arc) lo = mid; else hi = mid - 1;
+                }
+                j = lo;
+                v = __ldg(a.col + arc + s_delta[j]);
+                const int u = s_v[j];
+                const unsigned bit = 1u << (v & 31);
+                const unsigned vis = __ldcg(visited + (v >> 5));
+                if (MODE == XBFS_SF) {
+                    if (!(vis & bit)) {
+                        const unsigned old = atomicOr(visited + (v >> 5), bit);
+                        if (!(old & bit)) {
+                            win = true;
+                            level[v] = lvl;
+                            parent[v] = u;
+                            atomicOr(next + (v >> 5), bit);
+                            rs = a.row_ptr[v];
+                            deg = a.row_ptr[v + 1] - rs;
+                        }
+                    }
+                } else {
+                    // single-scan: the visited bitmap is stale only for this
+                    // level's own discoveries, which just repeat the same level
+                    // value (benign race; any writer's parent is valid, C-26).
+                    const unsigned nx = __ldcg(next + (v >> 5));
+                    if (!((vis | nx) & bit)) {
+                        level[v] = lvl;
+                        parent[v] = u;
+                        atomicOr(next + (v >> 5), bit);
+                    }
+                }
+            }
+            if (MODE == XBFS_SF)
+                enqueue_warp(win, v, rs, deg, &a.st->qctr[ob], a.dbits, a.qv[ob], a.qoff[ob], a.qdelta[ob],
+                             a.tile_first[ob]);
+        }
+    }
+}
+
+// -------------------------------------------------------------- generate
+// Bitmap -> queue (the single-scan generation pass, over the N-bit frontier
+// bitmap instead of the 4N-byte status array).  role 0: F_k from fb[k%3] into
+// queue k&1 (queue missing after a BU level).  role 1: F_{k+1} from
+// fb[(k+1)%3] into queue (k+1)&1 and visited |= F_{k+1} (after SS expansion).
+__global__ __launch_bounds__(kGenThreads) void k_generate(KArgs a, int role) {
+    count_launch(a.st);
+    const int k = a.st->k;
+    const unsigned int* __restrict__ bm = role == 0 ? a.fb[k % 3] : a.fb[(k + 1) % 3];
+    const int ob = role == 0 ? (k & 1) : ((k + 1) & 1);
+    unsigned long long* ctr = &a.st->qctr[ob];
+    const long long nth = (long long)gridDim.x * blockDim.x;
+    const long long base_tid = blockIdx.x * (long long)blockDim.x + (threadIdx.x & ~31);
+    const int lane = threadIdx.x & 31;
+    for (long long w0 = base_tid; w0 < a.words; w0 += nth) {
+        const long long w = w0 + lane;
+        unsigned word = w < a.words ? bm[w] : 0u;
+        if (role == 1 && word) a.visited[w] |= word;
+        // pass 1: count and degree sum of this lane's vertices
+        const int cnt = __popc(word);
+        long long dsum = 0;
+        for (unsigned b = word; b; b &= b - 1) {
+            const long long v = w * 32 + __ffs(b) - 1;
+            dsum += a.row_ptr[v + 1] - a.row_ptr[v];
+        }
+        int ic = cnt;
+        long long id = dsum;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const int tc = __shfl_up_sync(FULL, ic, o);
+            const long long td = __shfl_up_sync(FULL, id, o);
+            if (lane >= o) { ic += tc; id += td; }
+        }
+        const int wc = __shfl_sync(FULL, ic, 31);
+        if (wc == 0) continue;
+        const long long wd = __shfl_sync(FULL, id, 31);
+        unsigned long long base = 0;
+        if (lane == 0) base = atomicAdd(ctr, ((unsigned long long)wc << a.dbits) + (unsigned long long)wd);
+        base = __shfl_sync(FULL, base, 0);
+        long long slot = (long long)(base >> a.dbits) + ic - cnt;
+        long long off = (long long)(base & ((1ull << a.dbits) - 1ull)) + id - dsum;
+        int* qv = a.qv[ob];
+        long long* qoff = a.qoff[ob];
+        long long* qdelta = a.qdelta[ob];
+        int* tf = a.tile_first[ob];
+        for (unsigned b = word; b; b &= b - 1) {
+            const long long v = w * 32 + __ffs(b) - 1;
+            const long long rs = a.row_ptr[v], deg = a.row_ptr[v + 1] - rs;
+            qv[slot] = (int)v;
+            qoff[slot] = off;
+            qdelta[slot] = rs - off;
+            if (deg > 0) {
+                const long long t0 = (off + kTile - 1) / kTile, t1 = (off + deg - 1) / kTile;
+                for (long long t = t0; t <= t1; ++t) tf[t] = (int)slot;
+            }
+            ++slot;
+            off += deg;
+        }
+    }
+}
+
+// ------------------------------------------------------------- bottom-up
+// Candidates U_k = not visited (isolated vertices are pre-marked visited).
+// A candidate v is found iff some neighbour is in F_k = fb[k%3] (never a bit set
+// in this same pass: reading C-9), giving level k+1 and that neighbour as parent.
+__global__ __launch_bounds__(kBuThreads) void k_bu_traverse(KArgs a, int* __restrict__ level,
+                                                            int* __restrict__ parent) {
+    count_launch(a.st);
+    const int k = a.st->k;
+    clear_stale(a, k);
+    const unsigned int* __restrict__ cur = a.fb[k % 3];
+    unsigned int* __restrict__ next = a.fb[(k + 1) % 3];
+    const int lvl = k + 1;
+    const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+    __shared__ int s_list[kBuThreads / 32][1024];
+    __shared__ unsigned s_found[kBuThreads / 32][32];
+    const long long nchunks = (a.words + 31) / 32;
+    const long long gw = (blockIdx.x * (long long)blockDim.x + threadIdx.x) >> 5;
+    const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
+    unsigned long long found = 0, edges = 0, probes = 0;
+    for (long long c = gw; c < nchunks; c += nw) {
+        const long long w = c * 32 + lane;
+        const unsigned vis = w < a.words ? a.visited[w] : FULL;
+        const unsigned cand = ~vis;
+        const int cnt = __popc(cand);
+        int incl = cnt;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const int t = __shfl_up_sync(FULL, incl, o);
+            if (lane >= o) incl += t;
+        }
+        const int total = __shfl_sync(FULL, incl, 31);
+        int pos = incl - cnt;
+        for (unsigned b = cand; b; b &= b - 1) s_list[wib][pos++] = (int)(w * 32 + __ffs(b) - 1);
+        s_found[wib][lane] = 0;
+        __syncwarp();
+        for (int r = lane; r < total; r += 32) {
+            const int v = s_list[wib][r];
+            const long long rs = a.row_ptr[v], re = a.row_ptr[v + 1];
+            long long p = rs;
+            for (; p < re; ++p) {
+                const int u = __ldg(a.col + p);
+                if (__ldcg(cur + (u >> 5)) & (1u << (u & 31))) {
+                    level[v] = lvl;
+                    parent[v] = u;
+                    atomicOr(&s_found[wib][(v >> 5) - c * 32], 1u << (v & 31));
+                    edges += (unsigned long long)(re - rs);
+                    ++found;
+                    break;
+                }
+            }
+            probes += (unsigned long long)(p < re ? p - rs + 1 : re - rs);
+        }
+        __syncwarp();
+        if (w < a.words) {
+            const unsigned f = s_found[wib][lane];
+            next[w] = f;
+            if (f) a.visited[w] = vis | f;
+        }
+        __syncwarp();
+    }
+#pragma unroll
+    for (int o = 16; o; o >>= 1) {
+        found += __shfl_xor_sync(FULL, found, o);
+        edges += __shfl_xor_sync(FULL, edges, o);
+        probes += __shfl_xor_sync(FULL, probes, o);
+    }
+    if (lane == 0 && (found | edges | probes)) {
+        atomicAdd(&a.st->acc_found, found);
+        atomicAdd(&a.st->acc_edges, edges);
+        atomicAdd(&a.st->acc_probes, probes);
+    }
+}
+
+// ---------------------------------------------------------------- select
+__global__ void k_select(KArgs a) {
+    count_launch(a.st);
+    DevState* st = a.st;
+    const int k = st->k;
+    const int strat = st->strategy;
+    long long nf, ne;
+    if (strat == XBFS_BU) {
+        nf = (long long)st->acc_found;
+        ne = (long long)st->acc_edges;
+        st->queue_valid = 0;
+    } else {
+        const unsigned long long q = st->qctr[(k + 1) & 1];
+        nf = (long long)(q >> a.dbits);
+        ne = (long long)(q & ((1ull << a.dbits) - 1ull));
+        st->queue_valid = 1;
+    }
+    if (k < kLogCap) {
+        LevelRec r;
+        r.fsize = st->fsize;
+        r.fedges = st->fedges;
+        r.unvisited = st->unvisited;
+        r.probes = strat == XBFS_BU ? (long long)st->acc_probes : 0;
+        r.strategy = strat;
+        r.pad = 0;
+        a.log[k] = r;
+    }
+    st->reached += st->fsize;
+    st->arcs_traversed += st->fedges;
+    st->fprev = st->fsize;
+    st->fsize = nf;
+    st->fedges = ne;
+    st->unvisited -= nf;
+    st->acc_found = st->acc_edges = st->acc_probes = 0;
+    st->prev_strategy = strat;
+    st->k = k + 1;
+    if (nf == 0) {
+        st->done = 1;
+        st->nlevels = k + 1;
+    } else {
+        st->strategy = choose_strategy(st, a.arcs, nf, st->fprev, ne, st->unvisited, strat);
+        st->qctr[(k + 2) & 1] = 0;                   // queue buffer built during level k+1
+        if (!st->queue_valid) st->qctr[(k + 1) & 1] = 0;  // rebuilt by generate(role 0)
+    }
+    a.hctl->k = st->k;
+    a.hctl->strategy = st->strategy;
+    a.hctl->queue_valid = st->queue_valid;
+    a.hctl->done = st->done;
+}
+
+// Graph500 m (O-6) = sum of tuple counts over reached vertices; untimed.
+__global__ __launch_bounds__(256) void k_count_m(const int* __restrict__ level, const int* __restrict__ tcount,
+                                                 long long n, unsigned long long* out) {
+    unsigned long long s = 0;
+    for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < n;
+         v += (long long)gridDim.x * blockDim.x)
+        if (level[v] >= 0) s += (unsigned long long)tcount[v];
+    for (int o = 16; o; o >>= 1) s += __shfl_xor_sync(FULL, s, o);
+    if ((threadIdx.x & 31) == 0 && s) atomicAdd(out, s);
+}
+
+// ------------------------------------------------------------- drivers
+namespace {
+
+struct Grids {
+    int init, expand, gen, bu;
+};
+
+Grids grids_for(const xbfs_graph* g) {
+    Grids r;
+    r.init = g->num_sms * 8;
+    r.expand = g->num_sms * 4;   // 4 x 512 threads resident per SM
+    r.gen = g->num_sms * 8;
+    r.bu = g->num_sms * 8;       // 8 x 256 threads resident per SM
+    return r;
+}
+
+// Optional per-launch event timing (xbfs_run_stats.kernel_capacity > 0).
+struct Prof {
+    xbfs_graph* g = nullptr;
+    xbfs_run_stats* st = nullptr;
+    int n = 0;
+    bool on() const { return st && st->kernel_capacity > 0 && n < st->kernel_capacity; }
+    xbfs_status before() {
+        if (!on()) return XBFS_OK;
+        auto& ev = g->prof_events;
+        while ((int)ev.size() < 2 * (n + 1)) {
+            cudaEvent_t e;
+            XBFS_CUDA(g, cudaEventCreate(&e));
+            ev.push_back(e);
+        }
+        XBFS_CUDA(g, cudaEventRecord(ev[2 * n], g->stream));
+        return XBFS_OK;
+    }
+    xbfs_status after(int id, int level) {
+        if (!on()) return XBFS_OK;
+        XBFS_CUDA(g, cudaEventRecord(g->prof_events[2 * n + 1], g->stream));
+        if (st->kernel_id) st->kernel_id[n] = id;
+        if (st->kernel_level) st->kernel_level[n] = level;
+        ++n;
+        return XBFS_OK;
+    }
+    xbfs_status finish() {
+        if (!st || st->kernel_capacity <= 0) return XBFS_OK;
+        st->num_kernels = n;
+        for (int i = 0; i < n; ++i) {
+            float ms = 0.f;
+            XBFS_CUDA(g, cudaEventElapsedTime(&ms, g->prof_events[2 * i], g->prof_events[2 * i + 1]));
+            if (st->kernel_ms) st->kernel_ms[i] = ms;
+        }
+        return XBFS_OK;
+    }
+};
+
+#define XBFS_TRY(expr)                          \
+    do {                                        \
+        xbfs_status _s = (expr);                \
+        if (_s != XBFS_OK) return _s;           \
+    } while (0)
+
+#define XBFS_LAUNCH(prof, id, lvl, launch)      \
+    do {                                        \
+        XBFS_TRY((prof).before());              \
+        launch;                                 \
+        XBFS_CUDA((prof).g, cudaGetLastError()); \
+        XBFS_TRY((prof).after((id), (lvl)));    \
+    } while (0)
+
+// Enqueue one level given the host-known strategy / queue state.
+xbfs_status launch_level(xbfs_graph* g, const KArgs& a, int* level, int* parent, int k, int strat,
+                         int queue_valid, Prof& P) {
+    const Grids G = grids_for(g);
+    cudaStream_t s = g->stream;
+    if (strat != XBFS_BU && !queue_valid)
+        XBFS_LAUNCH(P, XBFS_K_GENERATE_PRE, k, (k_generate<<<G.gen, kGenThreads, 0, s>>>(a, 0)));
+    if (strat == XBFS_SF) {
+        XBFS_LAUNCH(P, XBFS_K_TD_SF, k,
+                    (k_td_expand<XBFS_SF><<<G.expand, kExpandThreads, 0, s>>>(a, level, parent)));
+    } else if (strat == XBFS_SS) {
+        XBFS_LAUNCH(P, XBFS_K_TD_SS, k,
+                    (k_td_expand<XBFS_SS><<<G.expand, kExpandThreads, 0, s>>>(a, level, parent)));
+        XBFS_LAUNCH(P, XBFS_K_GENERATE_POST, k, (k_generate<<<G.gen, kGenThreads, 0, s>>>(a, 1)));
+    } else {
+        XBFS_LAUNCH(P, XBFS_K_BU, k, (k_bu_traverse<<<G.bu, kBuThreads, 0, s>>>(a, level, parent)));
+    }
+    XBFS_LAUNCH(P, XBFS_K_SELECT, k, (k_select<<<1, 1, 0, s>>>(a)));
+    return XBFS_OK;
+}
+
+xbfs_status run_host_loop(xbfs_graph* g, const KArgs& a, int* level, int* parent, Prof& P) {
+    // k_seed wrote hctl; wait for it, then one sync per level (P:L151's
+    // host/device crossing, kept as the debug / measurement driver).
+    XBFS_CUDA(g, cudaStreamSynchronize(g->stream));
+    for (;;) {
+        volatile HostCtl* h = g->hctl;
+        if (h->done) break;
+        XBFS_TRY(launch_level(g, a, level, parent, h->k, h->strategy, h->queue_valid, P));
+        XBFS_CUDA(g, cudaStreamSynchronize(g->stream));
+    }
+    return XBFS_OK;
+}
+
+}  // namespace
+}  // namespace xbfs
+
+using namespace xbfs;
+
+static xbfs_status run_impl(xbfs_graph* g, int64_t source, int32_t* level, int32_t* parent,
+                            const xbfs_run_opts* opts, xbfs_run_stats* stats) {
+    if (!g) return set_error(XBFS_ERR_INVALID_ARG, "xbfs_run: NULL handle");
+    if (!level || !parent) return set_error(XBFS_ERR_INVALID_ARG, "xbfs_run: NULL level/parent");
+    if (source < 0 || source >= g->n)
+        return set_error(XBFS_ERR_INVALID_ARG, "xbfs_run: source %lld outside [0, %lld)", (long long)source, g->n);
+    if (g->poisoned) return set_error(XBFS_ERR_STATE, "handle poisoned by an earlier failure");
+    xbfs_run_opts o;
+    xbfs_run_opts_default(&o);
+    if (opts) o = *opts;
+    if (o.force_strategy < -1 || o.force_strategy > 2)
+        return set_error(XBFS_ERR_INVALID_ARG, "force_strategy must be -1..2");
+    XBFS_CUDA(g, cudaSetDevice(g->device));
+
+    KArgs a = g->kargs();
+    // selection parameters live in the device state
+    {
+        DevState hs;
+        memset(&hs, 0, sizeof(hs));
+        hs.alpha = o.alpha;
+        hs.grow = o.grow;
+        hs.ratio_min = o.ratio_min;
+        hs.bu_stay = o.bu_stay;
+        hs.force = o.force_strategy;
+        XBFS_CUDA(g, cudaMemcpyAsync(g->st, &hs, sizeof(hs), cudaMemcpyHostToDevice, g->stream));
+    }
+    const Grids G = grids_for(g);
+    Prof P;
+    P.g = g;
+    P.st = stats;
+    XBFS_CUDA(g, cudaEventRecord(g->ev0, g->stream));
+    XBFS_LAUNCH(P, XBFS_K_INIT, -1,
+                (k_init_fill<<<G.init, 256, 0, g->stream>>>(a, level, parent, g->nonisolated)));
+    XBFS_LAUNCH(P, XBFS_K_SEED, -1,
+                (k_seed<<<1, 1, 0, g->stream>>>(a, level, parent, source, g->nonisolated_count)));
+    XBFS_TRY(run_host_loop(g, a, level, parent, P));
+    XBFS_CUDA(g, cudaEventRecord(g->ev1, g->stream));
+
+    if (stats) {
+        XBFS_CUDA(g, cudaMemsetAsync(g->red_scratch, 0, sizeof(unsigned long long), g->stream));
+        k_count_m<<<G.init, 256, 0, g->stream>>>(level, g->tcount, g->n, g->red_scratch);
+        XBFS_CUDA(g, cudaGetLastError());
+        DevState hs;
+        unsigned long long m = 0;
+        XBFS_CUDA(g, cudaMemcpyAsync(&hs, g->st, sizeof(hs), cudaMemcpyDeviceToHost, g->stream));
+        XBFS_CUDA(g, cudaMemcpyAsync(&m, g->red_scratch, sizeof(m), cudaMemcpyDeviceToHost, g->stream));
+        XBFS_CUDA(g, cudaStreamSynchronize(g->stream));
+        float ms = 0.f;
+        XBFS_CUDA(g, cudaEventElapsedTime(&ms, g->ev0, g->ev1));
+        stats->elapsed_ms = ms;
+        stats->num_levels = hs.nlevels;
+        stats->vertices_reached = hs.reached;
+        stats->arcs_traversed = hs.arcs_traversed;
+        stats->input_edges_traversed = (int64_t)m;
+        stats->kernel_launches = hs.launches;
+        XBFS_TRY(P.finish());
+        const int nl = std::min(hs.nlevels, std::min(stats->level_capacity, kLogCap));
+        if (nl > 0 && (stats->strategy || stats->frontier_vertices || stats->frontier_edges ||
+                       stats->unvisited || stats->bu_probes)) {
+            LevelRec* rec = new LevelRec[nl];
+            XBFS_CUDA(g, cudaMemcpy(rec, g->log, nl * sizeof(LevelRec), cudaMemcpyDeviceToHost));
+            for (int i = 0; i < nl; ++i) {
+                if (stats->strategy) stats->strategy[i] = (int8_t)rec[i].strategy;
+                if (stats->frontier_vertices) stats->frontier_vertices[i] = rec[i].fsize;
+                if (stats->frontier_edges) stats->frontier_edges[i] = rec[i].fedges;
+                if (stats->unvisited) stats->unvisited[i] = rec[i].unvisited;
+                if (stats->bu_probes) stats->bu_probes[i] = rec[i].probes;
+            }
+            delete[] rec;
+        }
+    }
+    return XBFS_OK;
+}
+
+extern "C" xbfs_status xbfs_run(xbfs_graph* g, int64_t source, int32_t* level, int32_t* parent,
+                                const xbfs_run_opts* opts, xbfs_run_stats* stats) {
+    return run_impl(g, source, level, parent, opts, stats);
+}
+
+extern "C" xbfs_status xbfs_run_host(xbfs_graph* g, int64_t source, int32_t* level_host, int32_t* parent_host,
+                                     const xbfs_run_opts* opts, xbfs_run_stats* stats) {
+    if (!g) return set_error(XBFS_ERR_INVALID_ARG, "xbfs_run_host: NULL handle");
+    if (!level_host || !parent_host) return set_error(XBFS_ERR_INVALID_ARG, "xbfs_run_host: NULL level/parent");
+    if (g->poisoned) return set_error(XBFS_ERR_STATE, "handle poisoned by an earlier failure");
+    XBFS_CUDA(g, cudaSetDevice(g->device));
+    if (!g->scratch_level) {
+        XBFS_CUDA(g, cudaMalloc(&g->scratch_level, g->n * sizeof(int)));
+        XBFS_CUDA(g, cudaMalloc(&g->scratch_parent, g->n * sizeof(int)));
+    }
+    xbfs_status s = run_impl(g, source, g->scratch_level, g->scratch_parent, opts, stats);
+    if (s != XBFS_OK) return s;
+    XBFS_CUDA(g, cudaMemcpyAsync(level_host, g->scratch_level, g->n * sizeof(int), cudaMemcpyDeviceToHost, g->stream));
+    XBFS_CUDA(g, cudaMemcpyAsync(parent_host, g->scratch_parent, g->n * sizeof(int), cudaMemcpyDeviceToHost, g->stream));
+    XBFS_CUDA(g, cudaStreamSynchronize(g->stream));
+    return XBFS_OK;
+}

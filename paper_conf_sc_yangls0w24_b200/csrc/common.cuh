@@ -1,0 +1,130 @@
+// common.cuh — internal types of libxbfs (B200 / sm_100a).  Not part of the ABI.
+//
+// Layout in HBM:
+//   row_ptr  int64[N+1]   col int32[A]      (8-byte edge, 4-byte vertex ids)
+//   tcount   int32[N]     tuples per first endpoint (Graph500 m, O-6)
+//   visited  uint32[W]    W = ceil(N/32); isolated vertices pre-set (never candidates)
+//   fb[3]    uint32[W]    frontier bitmaps, rotated: level k reads fb[k%3] (F_k),
+//                         writes fb[(k+1)%3] (F_{k+1}), clears fb[(k+2)%3] (F_{k-1})
+//   queue[2] {qv int32, qoff int64, qdelta int64}[N] + tile_first int32[A/TILE+2]
+//            qoff = exclusive prefix of degrees over the queue (edge-balanced tiles),
+//            qdelta = row_ptr[v] - qoff, so arc a of the frontier is col[a + qdelta[j]].
+//   DevState (device) + HostCtl (pinned, mapped) per handle.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <vector>
+
+#include "xbfs.h"
+
+namespace xbfs {
+
+constexpr int kTile = 2048;          // frontier arcs per td_expand tile
+constexpr int kExpandThreads = 512;  // td_expand block
+constexpr int kBuThreads = 256;      // bu_traverse block (8 warps, 1024 vertices per warp chunk)
+constexpr int kGenThreads = 256;
+constexpr int kLogCap = 1 << 16;     // per-level log entries kept on the device
+
+struct LevelRec {
+    long long fsize, fedges, unvisited, probes;
+    int strategy, pad;
+};
+
+// Mirror of the scalars the host loop needs after each select (pinned + mapped).
+struct HostCtl {
+    int k, strategy, queue_valid, done;
+};
+
+struct DevState {
+    int k;                  // level being processed
+    int strategy;           // strategy chosen for level k
+    int queue_valid;        // queue buffer k&1 holds F_k
+    int done;
+    unsigned long long qctr[2];  // packed (count << dbits) + degree sum, per queue buffer
+    long long fsize, fedges;     // |F_k|, edgesF_k
+    long long fprev;             // |F_{k-1}|
+    long long unvisited;         // U_k (non-isolated, unvisited)
+    unsigned long long acc_found, acc_edges, acc_probes;  // BU accumulators for level k
+    long long reached, arcs_traversed;
+    unsigned int launches;       // library kernels launched (device-counted)
+    int nlevels;
+    // selection parameters (copied from xbfs_run_opts)
+    double alpha, grow, ratio_min, bu_stay;
+    int force, prev_strategy;
+    long long source;
+};
+
+// Arguments shared by all level kernels (static per handle => graph-capturable).
+struct KArgs {
+    const long long* row_ptr;
+    const int* col;
+    int* level;
+    int* parent;
+    unsigned int* visited;
+    unsigned int* fb[3];
+    int* qv[2];
+    long long* qoff[2];
+    long long* qdelta[2];
+    int* tile_first[2];
+    DevState* st;
+    HostCtl* hctl;          // device alias of the mapped host struct
+    LevelRec* log;
+    long long n;
+    long long words;        // ceil(N/32)
+    long long arcs;         // A
+    int dbits;              // low bits of qctr holding the degree sum
+};
+
+}  // namespace xbfs
+
+struct xbfs_graph {
+    int device = 0;
+    cudaStream_t stream = nullptr;
+    bool poisoned = false;
+    long long n = 0, arcs = 0, m_input = 0;
+    int max_deg = 0;
+    int reorder_mode = 0;
+    int num_sms = 148;
+    // CSR
+    long long* row_ptr = nullptr;
+    int* col = nullptr;
+    int* tcount = nullptr;
+    unsigned int* nonisolated = nullptr;
+    long long nonisolated_count = 0;
+    // BFS work state
+    unsigned int* visited = nullptr;
+    unsigned int* fb = nullptr;          // 3 * words
+    int* qv = nullptr;                   // 2 * N
+    long long* qoff = nullptr;           // 2 * N
+    long long* qdelta = nullptr;         // 2 * N
+    int* tile_first = nullptr;           // 2 * tiles_cap
+    long long tiles_cap = 0;
+    xbfs::DevState* st = nullptr;
+    xbfs::LevelRec* log = nullptr;
+    xbfs::HostCtl* hctl = nullptr;       // pinned host
+    xbfs::HostCtl* hctl_dev = nullptr;   // its device alias
+    unsigned long long* red_scratch = nullptr;  // reductions for stats
+    int* scratch_level = nullptr;        // xbfs_run_host device scratch
+    int* scratch_parent = nullptr;
+    cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+    int dbits = 40;
+    // CUDA-graph device loop (built lazily)
+    cudaGraphExec_t loop_exec = nullptr;
+    int* loop_level_ptr = nullptr;       // level/parent the graph was built for
+    int* loop_parent_ptr = nullptr;
+    std::vector<cudaEvent_t> prof_events;  // per-launch timing pool
+    xbfs::KArgs kargs() const;
+};
+
+namespace xbfs {
+// error plumbing (api.cu)
+xbfs_status set_error(xbfs_status s, const char* fmt, ...);
+xbfs_status cuda_fail(xbfs_graph* g, cudaError_t e, const char* what);
+}  // namespace xbfs
+
+#define XBFS_CUDA(g, call)                                                  \
+    do {                                                                    \
+        cudaError_t _e = (call);                                            \
+        if (_e != cudaSuccess) return ::xbfs::cuda_fail((g), _e, #call);    \
+    } while (0)

@@ -48,28 +48,39 @@ def quartiles(xs: Sequence[float]):
 # --------------------------------------------------------------------------
 # Algorithmic bytes per kernel launch.  Inputs are the per-level
 # counters the library logs; used for the bench's live roofline figure.
+# B = 4*ceil(n/32) bytes is one pass over an n-bit bitmap.  Bitmap probes per
+# arc are L2 traffic (the bitmaps are L2-resident) and are not counted.
 # --------------------------------------------------------------------------
 
-def bytes_td_expand(f_size: int, f_edges: int, found: int) -> int:
-    """Top-down expansion of F_k: 20 B per frontier queue entry (id + two
-    int64 offsets) + 4 B per expanded arc (col) + per discovered vertex 4 B
-    level + 4 B parent + 16 B row_ptr pair + 20 B next-queue entry (SF)."""
-    return 20 * f_size + 4 * f_edges + 44 * found
-
-
-def bytes_generate(n: int, f_size: int) -> int:
-    """Bitmap scan (n/8 B) + per frontier vertex 16 B row_ptr pair + 20 B queue
-    entry."""
-    return n // 8 + 36 * f_size
-
-
-def bytes_bu(n: int, unvisited: int, probes: int, found: int) -> int:
-    """Bottom-up step: visited + non-isolated words read (n/4 B), next and
-    visited words written (n/4 B), 16 B row_ptr pair per candidate, 4 B per
-    probed arc, 8 B level+parent per found vertex."""
-    return n // 4 + n // 4 + 16 * unvisited + 4 * probes + 8 * found
+def bitmap_bytes(n: int) -> int:
+    return 4 * ((n + 31) // 32)
 
 
 def bytes_init(n: int) -> int:
-    """level + parent fill (8n) and four n-bit bitmaps cleared."""
-    return 8 * n + 4 * ((n + 7) // 8)
+    """level + parent fill (8n) + visited write, non-isolated read, 3 frontier maps."""
+    return 8 * n + 5 * bitmap_bytes(n)
+
+
+def bytes_td_sf(n: int, f_size: int, f_edges: int, found: int) -> int:
+    """Scan-free expansion: stale-map clear + 20 B per queue entry (id + two int64)
+    + 4 B per arc (col) + 44 B per discovered vertex (level, parent, row_ptr pair,
+    next-queue entry)."""
+    return bitmap_bytes(n) + 20 * f_size + 4 * f_edges + 44 * found
+
+
+def bytes_td_ss(n: int, f_size: int, f_edges: int, found: int) -> int:
+    """Single-scan expansion: as SF but only level + parent per discovered vertex."""
+    return bitmap_bytes(n) + 20 * f_size + 4 * f_edges + 8 * found
+
+
+def bytes_generate(n: int, count: int, post: bool) -> int:
+    """Bitmap -> queue: bitmap read (+ visited OR when post) + 36 B per vertex
+    (row_ptr pair + queue entry)."""
+    return (2 if post else 1) * bitmap_bytes(n) + 36 * count
+
+
+def bytes_bu(n: int, unvisited: int, probes: int, found: int) -> int:
+    """Bottom-up step: 4 bitmap passes (visited read + write, next write, stale
+    clear) + 16 B row_ptr pair per candidate + 4 B per probed arc + 8 B
+    level+parent per found vertex."""
+    return 4 * bitmap_bytes(n) + 16 * unvisited + 4 * probes + 8 * found

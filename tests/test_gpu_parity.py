@@ -1,0 +1,194 @@
+"""GPU parity: the CUDA path (through the C ABI) against the oracle.
+
+Levels are unique (hop distances) and must match the oracle BIT-EXACTLY;
+parents are not unique and must pass Graph500 validation V1-V5 against the
+input tuples.  Every strategy is forced on every level
+(SF-only, SS-only, BU-only) besides the adaptive selector, so each kernel is
+checked on its own."""
+import numpy as np
+import pytest
+
+import oracle
+from paper_conf_sc_yangls0w24_b200 import synth
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+MODES = [dict(), dict(force_strategy=0), dict(force_strategy=1), dict(force_strategy=2),
+         dict(alpha=0.02), dict(alpha=0.3, grow=1.0, ratio_min=0.0), dict(bu_stay=4.0)]
+
+
+@pytest.fixture(scope="module")
+def xb():
+    from paper_conf_sc_yangls0w24_b200 import xbfs
+    return xbfs
+
+
+def _dev(a):
+    return torch.from_numpy(np.ascontiguousarray(a).view(np.int32)).cuda()
+
+
+def _check_run(g, og, src, dst, root, **opts):
+    level, parent, st = g.run(int(root), stats=True, **opts)
+    lv, pa = level.cpu().numpy(), parent.cpu().numpy()
+    ref, _, nl = oracle.bfs(og, int(root))
+    assert np.array_equal(lv, ref), f"levels differ (root {root}, opts {opts})"
+    assert oracle.validate(og, src, dst, int(root), lv, pa) == 0, f"validation failed (root {root}, {opts})"
+    # counters against the oracle's per-level facts
+    fs, fe = oracle.level_stats(og, ref)
+    assert st.num_levels == nl
+    assert st.frontier_vertices == fs.tolist()
+    assert st.frontier_edges == fe.tolist()
+    assert st.vertices_reached == int((ref >= 0).sum())
+    assert st.arcs_traversed == int(fe.sum())
+    assert st.input_edges_traversed == oracle.input_edges(src, ref)
+    if "force_strategy" in opts:
+        assert set(st.strategy) == {opts["force_strategy"]}
+    return st
+
+
+@pytest.mark.parametrize("scale", [10, 14])
+def test_csr_build_and_reorder_bit_exact(xb, scale):
+    src, dst, n = synth.kronecker(scale, seed=1)
+    og = oracle.build_csr(n, src, dst)
+    g = xb.Graph(_dev(src), _dev(dst), n, reorder=False)
+    rp, col = g.csr()
+    assert np.array_equal(rp, og.row_ptr) and np.array_equal(col, og.col)
+    assert g.arcs == og.arcs and g.max_degree == og.degree().max() and g.m_input == src.shape[0]
+    g.reorder(1)
+    rp2, col2 = g.csr()
+    ro = oracle.reorder(og)
+    assert np.array_equal(rp2, og.row_ptr) and np.array_equal(col2, ro.col)
+    g.reorder(1)                                  # idempotent
+    assert np.array_equal(g.csr()[1], ro.col)
+    g.reorder(0)                                  # back to id order
+    assert np.array_equal(g.csr()[1], og.col)
+    g.close()
+
+
+def test_csr_build_host_int64_edges(xb):
+    src, dst, n = synth.kronecker(11, seed=4)
+    og = oracle.build_csr(n, src, dst)
+    g = xb.Graph(src.astype(np.int64), dst.astype(np.int64), n, reorder=False)
+    rp, col = g.csr()
+    assert np.array_equal(rp, og.row_ptr) and np.array_equal(col, og.col)
+    g.close()
+
+
+@pytest.mark.parametrize("opts", MODES)
+def test_kronecker_s10_all_roots_all_strategies(xb, opts):
+    src, dst, n = synth.kronecker(10, seed=1)
+    og = oracle.build_csr(n, src, dst)
+    g = xb.Graph(_dev(src), _dev(dst), n)
+    for root in synth.roots(n, src, dst, 16, root_seed=2):
+        _check_run(g, og, src, dst, root, **opts)
+    g.close()
+
+
+@pytest.mark.parametrize("opts", MODES[:4])
+def test_kronecker_s16_strategies(xb, opts):
+    src, dst, n = synth.kronecker(16, seed=3)
+    og = oracle.build_csr(n, src, dst)
+    g = xb.Graph(_dev(src), _dev(dst), n)
+    for root in synth.roots(n, src, dst, 6, root_seed=5):
+        _check_run(g, og, src, dst, root, **opts)
+    g.close()
+
+
+def test_kronecker_s20_adaptive(xb):
+    src, dst, n = synth.kronecker(20, seed=1)
+    og = oracle.build_csr(n, src, dst)
+    g = xb.Graph(_dev(src), _dev(dst), n)
+    for root in synth.roots(n, src, dst, 8, root_seed=2):
+        st = _check_run(g, og, src, dst, root)
+        assert 2 in st.strategy     # a BU level happens on Kronecker s20 with alpha 0.1
+    for root in synth.roots(n, src, dst, 2, root_seed=9):
+        for f in (0, 1, 2):
+            _check_run(g, og, src, dst, root, force_strategy=f)
+    g.close()
+
+
+@pytest.mark.parametrize("perm", [0, 10])
+def test_grid_levels(xb, perm):
+    W = H = 32 if perm else 48
+    src, dst, n = synth.grid(W, H, seed=3, perm_scale=perm)
+    og = oracle.build_csr(n, src, dst)
+    g = xb.Graph(_dev(src), _dev(dst), n)
+    for root in (0, n // 2 + W // 2, n - 1, 17):
+        for opts in MODES[:4]:
+            _check_run(g, og, src, dst, root, **opts)
+    g.close()
+
+
+def test_edge_cases(xb):
+    # N not a multiple of 32; isolated vertices; 2-vertex component; self loops; duplicates
+    n = 77
+    e = [(i, i + 1) for i in range(30)] + [(40, 41)] + [(50, 50), (3, 4), (4, 3), (3, 4)] + \
+        [(60, j) for j in range(61, 77)]
+    src = np.array([a for a, _ in e], np.uint32)
+    dst = np.array([b for _, b in e], np.uint32)
+    og = oracle.build_csr(n, src, dst)
+    g = xb.Graph(_dev(src), _dev(dst), n)
+    for root in (0, 29, 40, 50, 33, 60, 76):      # 50: self-loop only (isolated); 33: isolated
+        for opts in MODES:
+            _check_run(g, og, src, dst, root, **opts)
+    g.close()
+
+
+def test_empty_and_tiny_graphs(xb):
+    for n, e in [(1, []), (5, []), (2, [(0, 1)]), (33, [(0, 32)])]:
+        src = np.array([a for a, _ in e], np.uint32)
+        dst = np.array([b for _, b in e], np.uint32)
+        og = oracle.build_csr(n, src, dst)
+        g = xb.Graph(_dev(src) if len(e) else src, _dev(dst) if len(e) else dst, n)
+        for root in range(n):
+            for opts in MODES[:4]:
+                _check_run(g, og, src, dst, root, **opts)
+        g.close()
+
+
+def test_hub_root_and_random_graphs(xb):
+    rng = np.random.default_rng(0)
+    n = 5000
+    hub = np.stack([np.zeros(4000, np.int64), rng.integers(1, n, 4000)], 1)
+    rnd = rng.integers(0, n, (20000, 2))
+    e = np.concatenate([hub, rnd]).astype(np.uint32)
+    src, dst = e[:, 0].copy(), e[:, 1].copy()
+    og = oracle.build_csr(n, src, dst)
+    g = xb.Graph(_dev(src), _dev(dst), n)
+    for root in (0, 1, 4999):
+        for opts in MODES:
+            _check_run(g, og, src, dst, root, **opts)
+    g.close()
+
+
+def test_run_host_matches_device(xb):
+    src, dst, n = synth.kronecker(12, seed=2)
+    og = oracle.build_csr(n, src, dst)
+    g = xb.Graph(_dev(src), _dev(dst), n)
+    root = int(synth.roots(n, src, dst, 1)[0])
+    lh = np.empty(n, np.int32)
+    ph = np.empty(n, np.int32)
+    st = g.run_host(root, lh, ph, stats=True)
+    ref, _, nl = oracle.bfs(og, root)
+    assert np.array_equal(lh, ref) and oracle.validate(og, src, dst, root, lh, ph) == 0
+    assert st.num_levels == nl
+    g.close()
+
+
+def test_errors(xb):
+    src, dst, n = synth.kronecker(8, seed=1)
+    g = xb.Graph(_dev(src), _dev(dst), n)
+    lv = torch.empty(n, dtype=torch.int32, device="cuda")
+    with pytest.raises(xb.XbfsError) as ei:
+        xb.xbfs_run(g.handle, n, lv, lv)
+    assert ei.value.status == xb.XBFS_ERR_INVALID_ARG
+    with pytest.raises(xb.XbfsError):
+        xb.xbfs_run(g.handle, -1, lv, lv)
+    bad = np.array([0, n], np.uint32)
+    with pytest.raises(xb.XbfsError) as ei:
+        xb.Graph(bad, bad, n)
+    assert ei.value.status == xb.XBFS_ERR_INVALID_ARG
+    # the handle still works after rejected arguments
+    level, parent, _ = g.run(int(src[0]))
+    g.close()

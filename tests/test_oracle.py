@@ -310,24 +310,28 @@ def test_selector_paper_rule_on_table3():
 
 
 def test_byte_replay_hand_computed():
-    """Path 0-1-2-3 from s=0 (n=4, A=6); strategies SF, BU, SF.
-    deg = [1,2,2,1]; F = {0},{1},{2},{3}.
-      init         8*4 + 4*ceil(4/8)=4                     = 36
-      L0 SF        20*1 + 4*1 + 28*1                       = 52
-      L1 BU        n/4=1 + n/8=0 + 16*U_1(=2: {2,3}) + 4*probes + 8*1
-                   probes: v2 row [1,3] (reordered by deg desc: 1 (deg 2) then 3) -> 1
-                           v3 row [2] -> no level-1 neighbour -> deg = 1   => 2
-                   = 1 + 0 + 32 + 8 + 8                     = 49
-      L2 SF        after BU: generate n/8=0 + 28*1; 20*1 + 4*2 + 28*1 = 84
-      L3 SF        20*1 + 4*1 + 0                           = 24
+    """Path 0-1-2-3 from s=0 (n=4, one bitmap word: B = 4 bytes), strategies
+    SF, BU, SF, SF.  deg = [1,2,2,1]; F = {0},{1},{2},{3}.
+      init      8*4 + 5*4                                        = 52
+      L0 SF     B + 20*|F0| + 4*edgesF0(1) + 44*|F1|              = 4+20+4+44   = 72
+      L1 BU     4B + 16*U1 + 4*probes + 8*|F2|, U1 = {2,3}
+                probes: v2's reordered row [1 (deg 2), 3 (deg 1)] -> 1
+                        v3's row [2]: no level-1 neighbour -> deg 1  => 2
+                                                                  = 16+32+8+8   = 64
+      L2 SF     rebuild queue after BU: B + 36*|F2| = 40; then
+                B + 20 + 4*edgesF2(2) + 44*|F3|                   = 40+4+20+8+44 = 116
+      L3 SF     B + 20 + 4*1 + 0                                  = 28
+    SS variant at L2: 40 + (4 + 20 + 8 + 8*1) + (8 + 36*1)       = 124
     """
     n, src, dst = _graph(4, [(0, 1), (1, 2), (2, 3)])
     g = oracle.reorder(oracle.build_csr(n, src, dst))
     level, _, nl = oracle.bfs(g, 0)
     assert nl == 4
     tot, per = oracle.byte_replay(g, level, [0, 2, 0, 0])
-    assert per.tolist() == [52, 49, 84, 24]
-    assert tot == 36 + 52 + 49 + 84 + 24
+    assert per.tolist() == [72, 64, 116, 28]
+    assert tot == 52 + 72 + 64 + 116 + 28
+    _, per2 = oracle.byte_replay(g, level, [0, 2, 1, 0])
+    assert per2[2] == 124
 
 
 # ------------------------------------------------------- paper byte model pin
