@@ -198,6 +198,10 @@ def run_ours(args):
     parent = torch.empty(n, dtype=torch.int32, device=dev)
     flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
     opts = dict(driver=args.driver)
+    if args.alpha is not None:
+        opts["alpha"] = args.alpha
+    if args.bu_stay is not None:
+        opts["bu_stay"] = args.bu_stay
 
     for r in warm:
         g.run(int(r), level, parent, stats=True, **opts)
@@ -240,6 +244,8 @@ def run_ours(args):
     lh = torch.empty(n, dtype=torch.int32, pin_memory=True).numpy()
     ph = torch.empty(n, dtype=torch.int32, pin_memory=True).numpy()
     e2e_t = []
+    if args.e2e_roots:
+        g.run_host(int(warm[0]), lh, ph, **opts)      # warm-up: instantiates the device loop for these buffers
     for r in mine[: min(len(mine), args.e2e_roots)]:
         flush.fill_(1)
         torch.cuda.synchronize()
@@ -311,7 +317,8 @@ def run_ours(args):
         "data": "synthetic (seeded Graph500 Kronecker generator, graph seed 1, root seed 2)",
         "config": {"workload": workload_name(args.config), "n_vertices": n, "input_edges": int(src.shape[0]),
                    "arcs": g.arcs, "roots_per_gpu": args.steps, "l2_flush": "512 MiB write before every timed BFS",
-                   "reorder": "degree-desc (P:L153)", "alpha": 0.1, "driver": args.driver,
+                   "reorder": "degree-desc (P:L153)", "alpha": opts.get("alpha", 0.1),
+                   "bu_stay": opts.get("bu_stay", 1.0), "driver": args.driver,
                    "parallelism": f"replicas x{world} (independent roots)"},
         "gteps_hmean_per_gpu": round(worst["hmean"] / 1e9, 3),
         "gteps_arcs_hmean": round(res["teps_arcs"] / 1e9, 3),
@@ -404,7 +411,9 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--config", default="s24", choices=sorted(CONFIGS))
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--driver", type=int, default=0, help="0 auto, 1 host loop, 2 CUDA-graph device loop")
+    ap.add_argument("--driver", type=int, default=1, help="0 auto, 1 host loop, 2 CUDA-graph device loop")
+    ap.add_argument("--alpha", type=float, default=None)
+    ap.add_argument("--bu-stay", type=float, default=None)
     ap.add_argument("--e2e-roots", type=int, default=8)
     ap.add_argument("--profile-roots", type=int, default=4)
     ap.add_argument("--cpu-budget", type=float, default=15.0)

@@ -63,7 +63,7 @@ typedef struct {
     double alpha;            /* BU iff edgesF_k / A > alpha; default 0.1 */
     double grow;             /* SS iff |F_k| > grow * |F_{k-1}| and ratio > ratio_min (C-10) */
     double ratio_min;        /*   "                                                    */
-    double bu_stay;          /* >0: stay BU while |U_k| * bu_stay < edgesF_k (C-11); 0 = off */
+    double bu_stay;          /* >0: stay BU while |U_k| * bu_stay < edgesF_k (C-11); default 1.0, 0 = paper rule */
     int32_t force_strategy;  /* -1 adaptive; 0 SF, 1 SS, 2 BU on every level (tests, Fig 7 sweep) */
     int32_t driver;          /* 0 auto, 1 host loop (one sync per level), 2 CUDA-graph device loop */
     int32_t lazy_init;       /* reserved (0) */
@@ -100,7 +100,7 @@ typedef struct {
 enum { XBFS_K_INIT = 0, XBFS_K_SEED = 1, XBFS_K_GENERATE_PRE = 2, XBFS_K_TD_SF = 3, XBFS_K_TD_SS = 4,
        XBFS_K_GENERATE_POST = 5, XBFS_K_BU = 6, XBFS_K_SELECT = 7 };
 
-/* Fill opts with the defaults (alpha 0.1, grow 2.0, ratio_min 1e-3, adaptive). */
+/* Fill opts with the defaults (alpha 0.1, grow 2.0, ratio_min 1e-3, bu_stay 1, adaptive). */
 void xbfs_run_opts_default(xbfs_run_opts* opts);
 
 /* Build the symmetric CSR (Graph500 "kernel 1"; P:L358 layout) from M input

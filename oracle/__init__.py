@@ -60,6 +60,8 @@ def lib():
         L.oracle_select.restype = i32
         L.oracle_byte_replay.argtypes = [i64, P, P, P, i32, P, P]
         L.oracle_byte_replay.restype = i64
+        L.oracle_bu_probes.argtypes = [i64, P, P, P, i32]
+        L.oracle_bu_probes.restype = i64
         _lib = L
     return _lib
 
@@ -156,3 +158,9 @@ def byte_replay(g: CSR, level, strategy):
     tot = lib().oracle_byte_replay(g.n, _p(g.row_ptr), _p(g.col), _p(level), len(strategy),
                                    _p(strategy), _p(per))
     return int(tot), per[: len(strategy)].copy()
+
+
+def bu_probes(g: CSR, level, k: int) -> int:
+    """Arcs probed by a bottom-up step at level k with early termination."""
+    level = np.ascontiguousarray(level, dtype=np.int32)
+    return int(lib().oracle_bu_probes(g.n, _p(g.row_ptr), _p(g.col), _p(level), int(k)))

@@ -273,3 +273,20 @@ int64_t oracle_byte_replay(int64_t n, const int64_t* row_ptr, const int32_t* col
     free(fsize); free(fedges);
     return total;
 }
+
+/* Arcs a bottom-up step at level k probes (P:L124-131 early termination): over
+ * the candidates (non-isolated, not reached by level k), 1 + index of the first
+ * neighbour at level k in the stored row, or the whole degree if none. */
+int64_t oracle_bu_probes(int64_t n, const int64_t* row_ptr, const int32_t* col,
+                         const int32_t* level, int32_t k) {
+    int64_t probes = 0;
+    for (int64_t v = 0; v < n; ++v) {
+        if (row_ptr[v + 1] == row_ptr[v]) continue;
+        if (level[v] >= 0 && level[v] <= k) continue;
+        int64_t pr = row_ptr[v + 1] - row_ptr[v];
+        for (int64_t p = row_ptr[v]; p < row_ptr[v + 1]; ++p)
+            if (level[col[p]] == k) { pr = p - row_ptr[v] + 1; break; }
+        probes += pr;
+    }
+    return probes;
+}

@@ -36,7 +36,8 @@ xbfs::KArgs xbfs_graph::kargs() const {
     a.level = nullptr;
     a.parent = nullptr;
     a.visited = visited;
-    for (int i = 0; i < 3; ++i) a.fb[i] = fb + i * words;
+    const long long stride = (words + 31) / 32 * 32;  // 128-byte aligned bitmaps (uint4 access)
+    for (int i = 0; i < 3; ++i) a.fb[i] = fb + i * stride;
     for (int i = 0; i < 2; ++i) {
         a.qv[i] = qv + i * n;
         a.qoff[i] = qoff + i * n;
@@ -71,7 +72,7 @@ void xbfs_run_opts_default(xbfs_run_opts* o) {
     o->alpha = 0.1;
     o->grow = 2.0;        // reading C-10
     o->ratio_min = 1e-3;  // reading C-10
-    o->bu_stay = 0.0;     // reading C-11 (off = paper rule)
+    o->bu_stay = 1.0;     // reading C-11, tuned on B200 (tools/sweep_selector.py); 0 = paper rule
     o->force_strategy = -1;
     o->driver = 0;
 }
@@ -105,7 +106,7 @@ void xbfs_destroy(xbfs_graph* g) {
     if (!g) return;
     cudaSetDevice(g->device);
     if (g->stream) cudaStreamSynchronize(g->stream);
-    if (g->loop_exec) cudaGraphExecDestroy(g->loop_exec);
+    g->drop_loops();
     void* dev[] = {g->row_ptr, g->col, g->tcount, g->nonisolated, g->visited, g->fb, g->qv,
                    g->qoff, g->qdelta, g->tile_first, g->st, g->log, g->red_scratch,
                    g->scratch_level, g->scratch_parent};

@@ -121,9 +121,10 @@ __device__ int choose_strategy(const DevState* st, long long arcs, long long fsi
 }
 
 // Seed the source (the source holds level 0) and reset the level state.
-__global__ void k_seed(KArgs a, int* level, int* parent, long long s, long long nonisolated_count) {
+__global__ void k_seed(KArgs a, int* level, int* parent, long long nonisolated_count) {
     count_launch(a.st);
     DevState* st = a.st;
+    const long long s = st->source;   // per-run parameter copied in before init
     const long long rs = a.row_ptr[s], deg = a.row_ptr[s + 1] - rs;
     level[s] = 0;
     parent[s] = (int)s;
@@ -325,15 +326,22 @@ __global__ __launch_bounds__(kBuThreads) void k_bu_traverse(KArgs a, int* __rest
     unsigned int* __restrict__ next = a.fb[(k + 1) % 3];
     const int lvl = k + 1;
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
-    __shared__ int s_list[kBuThreads / 32][1024];
-    __shared__ unsigned s_found[kBuThreads / 32][32];
-    const long long nchunks = (a.words + 31) / 32;
+    const unsigned lt = (1u << lane) - 1u;
+    constexpr int kCW = kBuChunkWords, kCV = kBuChunkWords * 32;
+    __shared__ int s_list[kBuThreads / 32][kCV];   // candidates of the warp's chunk
+    __shared__ int s_hard[kBuThreads / 32][kCV];   // long unresolved rows (warp-cooperative)
+    __shared__ int s_hoff[kBuThreads / 32][kCV];   // arcs already probed for each hard row
+    __shared__ unsigned s_found[kBuThreads / 32][kCW];
+    const long long nchunks = (a.words + kCW - 1) / kCW;
     const long long gw = (blockIdx.x * (long long)blockDim.x + threadIdx.x) >> 5;
     const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
     unsigned long long found = 0, edges = 0, probes = 0;
     for (long long c = gw; c < nchunks; c += nw) {
-        const long long w = c * 32 + lane;
-        const unsigned vis = w < a.words ? a.visited[w] : FULL;
+        // 1. candidates of kCW bitmap words: ballot/popc compaction into shared memory
+        //    (the paper's count + prefix-sum + queue-write "double scan").
+        const long long w = c * kCW + lane;
+        const bool own = lane < kCW && w < a.words;
+        const unsigned vis = own ? a.visited[w] : FULL;
         const unsigned cand = ~vis;
         const int cnt = __popc(cand);
         int incl = cnt;
@@ -345,27 +353,96 @@ __global__ __launch_bounds__(kBuThreads) void k_bu_traverse(KArgs a, int* __rest
         const int total = __shfl_sync(FULL, incl, 31);
         int pos = incl - cnt;
         for (unsigned b = cand; b; b &= b - 1) s_list[wib][pos++] = (int)(w * 32 + __ffs(b) - 1);
-        s_found[wib][lane] = 0;
+        if (lane < kCW) s_found[wib][lane] = 0;
         __syncwarp();
-        for (int r = lane; r < total; r += 32) {
-            const int v = s_list[wib][r];
-            const long long rs = a.row_ptr[v], re = a.row_ptr[v + 1];
-            long long p = rs;
-            for (; p < re; ++p) {
-                const int u = __ldg(a.col + p);
-                if (__ldcg(cur + (u >> 5)) & (1u << (u & 31))) {
+        // 2. lane-per-candidate, kBuBatch arcs per step in stored (degree-desc) order;
+        //    a lane that finishes takes the next candidate, so lanes stay busy.
+        int v = -1, nxt = 0, nhard = 0;
+        long long rs = 0, re = 0, p = 0;
+        for (;;) {
+            const unsigned need = __ballot_sync(FULL, v < 0);
+            if (v < 0) {
+                const int idx = nxt + __popc(need & lt);
+                if (idx < total) {
+                    v = s_list[wib][idx];
+                    rs = a.row_ptr[v];
+                    re = a.row_ptr[v + 1];
+                    p = rs;
+                }
+            }
+            nxt += __popc(need);
+            if (!__any_sync(FULL, v >= 0)) break;
+            bool to_hard = false;
+            if (v >= 0) {
+                const long long end = min(re, p + kBuBatch);
+                int u[kBuBatch];
+                unsigned wd[kBuBatch];
+#pragma unroll
+                for (int j = 0; j < kBuBatch; ++j) u[j] = (p + j < end) ? __ldg(a.col + p + j) : -1;
+#pragma unroll
+                for (int j = 0; j < kBuBatch; ++j) wd[j] = u[j] >= 0 ? __ldcg(cur + (u[j] >> 5)) : 0u;
+                int hit = -1;
+#pragma unroll
+                for (int j = kBuBatch - 1; j >= 0; --j)
+                    if (u[j] >= 0 && ((wd[j] >> (u[j] & 31)) & 1u)) hit = j;   // first hit in row order
+                if (hit >= 0) {
+                    int pu = u[0];
+#pragma unroll
+                    for (int j = 1; j < kBuBatch; ++j) if (j == hit) pu = u[j];
                     level[v] = lvl;
-                    parent[v] = u;
-                    atomicOr(&s_found[wib][(v >> 5) - c * 32], 1u << (v & 31));
+                    parent[v] = pu;
+                    atomicOr(&s_found[wib][(v >> 5) - c * kCW], 1u << (v & 31));
                     edges += (unsigned long long)(re - rs);
                     ++found;
+                    probes += (unsigned long long)(p + hit + 1 - rs);
+                    v = -1;
+                } else if (end == re) {
+                    probes += (unsigned long long)(re - rs);
+                    v = -1;
+                } else if (re - end > kBuHardMin) {
+                    to_hard = true;
+                } else {
+                    p = end;
+                }
+            }
+            const unsigned hm = __ballot_sync(FULL, to_hard);
+            if (to_hard) {
+                const int hi = nhard + __popc(hm & lt);
+                s_hard[wib][hi] = v;
+                s_hoff[wib][hi] = (int)(p + kBuBatch - rs);
+                v = -1;
+            }
+            nhard += __popc(hm);
+        }
+        __syncwarp();
+        // 3. long unresolved rows: the whole warp probes 32 arcs per step, first hit wins
+        for (int h = 0; h < nhard; ++h) {
+            const int hv = s_hard[wib][h];
+            const long long hrs = a.row_ptr[hv], hre = a.row_ptr[hv + 1];
+            bool hit_any = false;
+            for (long long base = hrs + s_hoff[wib][h]; base < hre; base += 32) {
+                const long long pp = base + lane;
+                const int u = pp < hre ? __ldg(a.col + pp) : -1;
+                const bool hit = u >= 0 && ((__ldcg(cur + (u >> 5)) >> (u & 31)) & 1u);
+                const unsigned m = __ballot_sync(FULL, hit);
+                if (m) {
+                    const int first = __ffs(m) - 1;
+                    if (lane == first) {
+                        level[hv] = lvl;
+                        parent[hv] = u;
+                        atomicOr(&s_found[wib][(hv >> 5) - c * kCW], 1u << (hv & 31));
+                        edges += (unsigned long long)(hre - hrs);
+                        ++found;
+                        probes += (unsigned long long)(pp + 1 - hrs);
+                    }
+                    hit_any = true;
                     break;
                 }
             }
-            probes += (unsigned long long)(p < re ? p - rs + 1 : re - rs);
+            if (!hit_any && lane == 0) probes += (unsigned long long)(hre - hrs);
         }
         __syncwarp();
-        if (w < a.words) {
+        if (own) {
             const unsigned f = s_found[wib][lane];
             next[w] = f;
             if (f) a.visited[w] = vis | f;
@@ -386,7 +463,8 @@ __global__ __launch_bounds__(kBuThreads) void k_bu_traverse(KArgs a, int* __rest
 }
 
 // ---------------------------------------------------------------- select
-__global__ void k_select(KArgs a) {
+template <bool kGraph>
+__global__ void k_select(KArgs a, cudaGraphConditionalHandle h_while) {
     count_launch(a.st);
     DevState* st = a.st;
     const int k = st->k;
@@ -433,6 +511,15 @@ __global__ void k_select(KArgs a) {
     a.hctl->strategy = st->strategy;
     a.hctl->queue_valid = st->queue_valid;
     a.hctl->done = st->done;
+    if (kGraph) cudaGraphSetConditional(h_while, st->done ? 0u : 1u);
+}
+
+// Device loop: map (strategy, queue_valid) of level k to a SWITCH branch.
+__global__ void k_plan(KArgs a, cudaGraphConditionalHandle h_switch) {
+    count_launch(a.st);
+    const int s = a.st->strategy, qv = a.st->queue_valid;
+    const unsigned br = s == XBFS_BU ? 4u : (s == XBFS_SF ? (qv ? 0u : 1u) : (qv ? 2u : 3u));
+    cudaGraphSetConditional(h_switch, br);
 }
 
 // Graph500 m (O-6) = sum of tuple counts over reached vertices; untimed.
@@ -530,7 +617,7 @@ xbfs_status launch_level(xbfs_graph* g, const KArgs& a, int* level, int* parent,
     } else {
         XBFS_LAUNCH(P, XBFS_K_BU, k, (k_bu_traverse<<<G.bu, kBuThreads, 0, s>>>(a, level, parent)));
     }
-    XBFS_LAUNCH(P, XBFS_K_SELECT, k, (k_select<<<1, 1, 0, s>>>(a)));
+    XBFS_LAUNCH(P, XBFS_K_SELECT, k, (k_select<false><<<1, 1, 0, s>>>(a, 0)));
     return XBFS_OK;
 }
 
@@ -544,6 +631,105 @@ xbfs_status run_host_loop(xbfs_graph* g, const KArgs& a, int* level, int* parent
         XBFS_TRY(launch_level(g, a, level, parent, h->k, h->strategy, h->queue_valid, P));
         XBFS_CUDA(g, cudaStreamSynchronize(g->stream));
     }
+    return XBFS_OK;
+}
+
+// ------------------------------------------------- CUDA-graph device loop
+// One graph per (handle, level, parent): init -> seed -> WHILE(!done) {
+//   plan -> SWITCH{SF | gen+SF | SS+gen | gen+SS+gen | BU} -> select }.
+// The strategy decision never leaves the device: one launch per BFS instead of
+// one host/device crossing per level (the paper's P:L151 cost).
+xbfs_status add_kernel(xbfs_graph* g, cudaGraph_t gr, cudaGraphNode_t* out, const cudaGraphNode_t* dep,
+                       void* fn, int grid, int block, void** args) {
+    cudaKernelNodeParams p = {};
+    p.func = fn;
+    p.gridDim = dim3(grid);
+    p.blockDim = dim3(block);
+    p.sharedMemBytes = 0;
+    p.kernelParams = args;
+    p.extra = nullptr;
+    XBFS_CUDA(g, cudaGraphAddKernelNode(out, gr, dep, dep ? 1 : 0, &p));
+    return XBFS_OK;
+}
+
+xbfs_status build_loop_graph(xbfs_graph* g, int* level, int* parent) {
+    xbfs_graph::LoopGraph* slot = &g->loops[0];
+    for (auto& l : g->loops) {
+        if (l.exec && l.level == level && l.parent == parent) {
+            l.used = ++g->loop_tick;
+            g->cur_exec = l.exec;
+            return XBFS_OK;
+        }
+        if (l.used < slot->used) slot = &l;
+    }
+    if (slot->exec) { cudaGraphExecDestroy(slot->exec); *slot = xbfs_graph::LoopGraph(); }
+    const Grids G = grids_for(g);
+    KArgs a = g->kargs();
+    const unsigned int* noniso = g->nonisolated;
+    long long nic = g->nonisolated_count;
+    cudaGraph_t top = nullptr;
+    XBFS_CUDA(g, cudaGraphCreate(&top, 0));
+    struct Del { cudaGraph_t& t; ~Del() { if (t) cudaGraphDestroy(t); } } del{top};
+    cudaGraphNode_t n_init, n_seed, n_while, n_plan, n_sw, n_sel, x, y;
+    {
+        void* args[] = {&a, &level, &parent, &noniso};
+        XBFS_TRY(add_kernel(g, top, &n_init, nullptr, (void*)k_init_fill, G.init, 256, args));
+    }
+    {
+        void* args[] = {&a, &level, &parent, &nic};
+        XBFS_TRY(add_kernel(g, top, &n_seed, &n_init, (void*)k_seed, 1, 1, args));
+    }
+    cudaGraphConditionalHandle h_while, h_switch;
+    XBFS_CUDA(g, cudaGraphConditionalHandleCreate(&h_while, top, 1, cudaGraphCondAssignDefault));
+    cudaGraphNodeParams wp = {};
+    wp.type = cudaGraphNodeTypeConditional;
+    wp.conditional.handle = h_while;
+    wp.conditional.type = cudaGraphCondTypeWhile;
+    wp.conditional.size = 1;
+    XBFS_CUDA(g, cudaGraphAddNode(&n_while, top, &n_seed, 1, &wp));
+    cudaGraph_t body = wp.conditional.phGraph_out[0];
+    XBFS_CUDA(g, cudaGraphConditionalHandleCreate(&h_switch, body, 0, cudaGraphCondAssignDefault));
+    {
+        void* args[] = {&a, &h_switch};
+        XBFS_TRY(add_kernel(g, body, &n_plan, nullptr, (void*)k_plan, 1, 1, args));
+    }
+    cudaGraphNodeParams sp = {};
+    sp.type = cudaGraphNodeTypeConditional;
+    sp.conditional.handle = h_switch;
+    sp.conditional.type = cudaGraphCondTypeSwitch;
+    sp.conditional.size = 5;
+    XBFS_CUDA(g, cudaGraphAddNode(&n_sw, body, &n_plan, 1, &sp));
+    cudaGraph_t* br = sp.conditional.phGraph_out;
+    int role0 = 0, role1 = 1;
+    void* a_exp[] = {&a, &level, &parent};
+    void* a_gen0[] = {&a, &role0};
+    void* a_gen1[] = {&a, &role1};
+    void* f_sf = (void*)k_td_expand<XBFS_SF>;
+    void* f_ss = (void*)k_td_expand<XBFS_SS>;
+    void* f_gen = (void*)k_generate;
+    // 0: SF (queue valid)
+    XBFS_TRY(add_kernel(g, br[0], &x, nullptr, f_sf, G.expand, kExpandThreads, a_exp));
+    // 1: generate + SF
+    XBFS_TRY(add_kernel(g, br[1], &x, nullptr, f_gen, G.gen, kGenThreads, a_gen0));
+    XBFS_TRY(add_kernel(g, br[1], &y, &x, f_sf, G.expand, kExpandThreads, a_exp));
+    // 2: SS + generate (No-Frontier-Generation: the queue exists)
+    XBFS_TRY(add_kernel(g, br[2], &x, nullptr, f_ss, G.expand, kExpandThreads, a_exp));
+    XBFS_TRY(add_kernel(g, br[2], &y, &x, f_gen, G.gen, kGenThreads, a_gen1));
+    // 3: generate + SS + generate
+    XBFS_TRY(add_kernel(g, br[3], &x, nullptr, f_gen, G.gen, kGenThreads, a_gen0));
+    XBFS_TRY(add_kernel(g, br[3], &y, &x, f_ss, G.expand, kExpandThreads, a_exp));
+    XBFS_TRY(add_kernel(g, br[3], &x, &y, f_gen, G.gen, kGenThreads, a_gen1));
+    // 4: BU
+    XBFS_TRY(add_kernel(g, br[4], &x, nullptr, (void*)k_bu_traverse, G.bu, kBuThreads, a_exp));
+    {
+        void* args[] = {&a, &h_while};
+        XBFS_TRY(add_kernel(g, body, &n_sel, &n_sw, (void*)k_select<true>, 1, 1, args));
+    }
+    XBFS_CUDA(g, cudaGraphInstantiate(&slot->exec, top, 0));
+    slot->level = level;
+    slot->parent = parent;
+    slot->used = ++g->loop_tick;
+    g->cur_exec = slot->exec;
     return XBFS_OK;
 }
 
@@ -576,19 +762,28 @@ static xbfs_status run_impl(xbfs_graph* g, int64_t source, int32_t* level, int32
         hs.ratio_min = o.ratio_min;
         hs.bu_stay = o.bu_stay;
         hs.force = o.force_strategy;
+        hs.source = source;
         XBFS_CUDA(g, cudaMemcpyAsync(g->st, &hs, sizeof(hs), cudaMemcpyHostToDevice, g->stream));
     }
     const Grids G = grids_for(g);
     Prof P;
     P.g = g;
     P.st = stats;
+    const bool use_graph = (o.driver == 0 || o.driver == 2) && !(stats && stats->kernel_capacity > 0);
+    if (use_graph) {
+        XBFS_TRY(build_loop_graph(g, level, parent));
+        XBFS_CUDA(g, cudaEventRecord(g->ev0, g->stream));
+        XBFS_CUDA(g, cudaGraphLaunch(g->cur_exec, g->stream));
+        XBFS_CUDA(g, cudaEventRecord(g->ev1, g->stream));
+    } else {
     XBFS_CUDA(g, cudaEventRecord(g->ev0, g->stream));
     XBFS_LAUNCH(P, XBFS_K_INIT, -1,
                 (k_init_fill<<<G.init, 256, 0, g->stream>>>(a, level, parent, g->nonisolated)));
     XBFS_LAUNCH(P, XBFS_K_SEED, -1,
-                (k_seed<<<1, 1, 0, g->stream>>>(a, level, parent, source, g->nonisolated_count)));
+                (k_seed<<<1, 1, 0, g->stream>>>(a, level, parent, g->nonisolated_count)));
     XBFS_TRY(run_host_loop(g, a, level, parent, P));
     XBFS_CUDA(g, cudaEventRecord(g->ev1, g->stream));
+    }
 
     if (stats) {
         XBFS_CUDA(g, cudaMemsetAsync(g->red_scratch, 0, sizeof(unsigned long long), g->stream));

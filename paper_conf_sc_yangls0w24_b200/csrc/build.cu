@@ -159,7 +159,7 @@ xbfs_status alloc_work(xbfs_graph* g) {
     const long long n = g->n, words = (n + 31) / 32;
     g->tiles_cap = g->arcs / kTile + 4;
     XBFS_CUDA(g, cudaMalloc(&g->visited, words * sizeof(unsigned int)));
-    XBFS_CUDA(g, cudaMalloc(&g->fb, 3 * words * sizeof(unsigned int)));
+    XBFS_CUDA(g, cudaMalloc(&g->fb, 3 * ((words + 31) / 32 * 32) * sizeof(unsigned int)));
     XBFS_CUDA(g, cudaMalloc(&g->qv, 2 * n * sizeof(int)));
     XBFS_CUDA(g, cudaMalloc(&g->qoff, 2 * n * sizeof(long long)));
     XBFS_CUDA(g, cudaMalloc(&g->qdelta, 2 * n * sizeof(long long)));
@@ -355,7 +355,7 @@ extern "C" xbfs_status xbfs_reorder(xbfs_graph* g, int32_t mode) {
     cudaFree(k0);
     cudaFree(k1);
     // the BFS graph (if any) captured the old col pointer
-    if (g->loop_exec) { cudaGraphExecDestroy(g->loop_exec); g->loop_exec = nullptr; }
+    g->drop_loops();
     g->reorder_mode = mode;
     return XBFS_OK;
 }

@@ -22,7 +22,10 @@ namespace xbfs {
 
 constexpr int kTile = 2048;          // frontier arcs per td_expand tile
 constexpr int kExpandThreads = 512;  // td_expand block
-constexpr int kBuThreads = 256;      // bu_traverse block (8 warps, 1024 vertices per warp chunk)
+constexpr int kBuThreads = 256;      // bu_traverse block (8 warps)
+constexpr int kBuChunkWords = 8;     // bitmap words (256 vertices) per warp chunk
+constexpr int kBuBatch = 8;          // arcs probed per lane step (one 32-byte sector of col)
+constexpr int kBuHardMin = 256;      // unresolved rows with more arcs left go warp-cooperative
 constexpr int kGenThreads = 256;
 constexpr int kLogCap = 1 << 16;     // per-level log entries kept on the device
 
@@ -110,9 +113,21 @@ struct xbfs_graph {
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
     int dbits = 40;
     // CUDA-graph device loop (built lazily)
-    cudaGraphExec_t loop_exec = nullptr;
-    int* loop_level_ptr = nullptr;       // level/parent the graph was built for
-    int* loop_parent_ptr = nullptr;
+    struct LoopGraph {
+        cudaGraphExec_t exec = nullptr;
+        int* level = nullptr;            // output pointers the graph was built for
+        int* parent = nullptr;
+        unsigned long long used = 0;
+    };
+    LoopGraph loops[4];                  // small LRU cache of instantiated device loops
+    unsigned long long loop_tick = 0;
+    cudaGraphExec_t cur_exec = nullptr;
+    void drop_loops() {
+        for (auto& l : loops) {
+            if (l.exec) cudaGraphExecDestroy(l.exec);
+            l = LoopGraph();
+        }
+    }
     std::vector<cudaEvent_t> prof_events;  // per-launch timing pool
     xbfs::KArgs kargs() const;
 };

@@ -15,7 +15,8 @@ torch = pytest.importorskip("torch")
 pytestmark = pytest.mark.gpu
 
 MODES = [dict(), dict(force_strategy=0), dict(force_strategy=1), dict(force_strategy=2),
-         dict(alpha=0.02), dict(alpha=0.3, grow=1.0, ratio_min=0.0), dict(bu_stay=4.0)]
+         dict(alpha=0.02), dict(alpha=0.3, grow=1.0, ratio_min=0.0), dict(bu_stay=4.0),
+         dict(driver=1), dict(driver=1, force_strategy=1), dict(driver=1, force_strategy=2)]
 
 
 @pytest.fixture(scope="module")
@@ -191,4 +192,28 @@ def test_errors(xb):
     assert ei.value.status == xb.XBFS_ERR_INVALID_ARG
     # the handle still works after rejected arguments
     level, parent, _ = g.run(int(src[0]))
+    g.close()
+
+
+@pytest.mark.parametrize("scale", [12, 16])
+def test_bu_probes_and_parents_match_definition(xb, scale):
+    """Bottom-up with early termination over degree-ordered rows
+    (P:L153): the GPU's per-level probe count equals the oracle's definition,
+    and a BU parent is exactly the first stored neighbour one level up."""
+    src, dst, n = synth.kronecker(scale, seed=7)
+    og = oracle.build_csr(n, src, dst)
+    ro = oracle.reorder(og)
+    g = xb.Graph(_dev(src), _dev(dst), n)
+    for root in synth.roots(n, src, dst, 3, root_seed=11):
+        for opts in (dict(force_strategy=2), dict(), dict(alpha=0.01)):
+            level, parent, st = g.run(int(root), stats=True, **opts)
+            ref, _, nl = oracle.bfs(og, int(root))
+            lv, pa = level.cpu().numpy(), parent.cpu().numpy()
+            assert np.array_equal(lv, ref)
+            for k in range(nl):
+                if st.strategy[k] == 2:
+                    assert st.bu_probes[k] == oracle.bu_probes(ro, ref, k), (k, opts)
+                    for v in np.flatnonzero(ref == k + 1)[:3000]:
+                        row = ro.col[ro.row_ptr[v]:ro.row_ptr[v + 1]]
+                        assert pa[v] == row[np.argmax(ref[row] == k)]
     g.close()

@@ -360,3 +360,23 @@ def test_harmonic_mean_and_quartiles():
     assert metrics.harmonic_mean([1.0, 2.0, 4.0]) == pytest.approx(3 / (1 + 0.5 + 0.25))
     q = metrics.quartiles([1, 2, 3, 4, 5])
     assert (q["min"], q["q1"], q["median"], q["q3"], q["max"]) == (1, 2, 3, 4, 5)
+
+
+def test_bu_probes_hand_computed():
+    """Star centre 0 with leaves 1..4 plus path 4-5-6, from s = 1.
+    levels: 1:0, 0:1, 2/3/4:2, 5:3, 6:4.  Reordered rows (deg desc, id asc):
+      0: [1,2,3,4] (all deg 1 except 4 with deg 2) -> [4,1,2,3];  4: [0,5] (deg 4, 2);
+      5: [4,6] (deg 2, 1); 6: [5].
+    BU at k=1 (candidates: 2,3,4,5,6): v2 row [0] hit at 1; v3 same 1; v4 row [0,5]: 0 hit -> 1;
+      v5 row [4,6]: no level-1 neighbour -> 2; v6 row [5] -> 1.  Total 6.
+    BU at k=2 (candidates 5,6): v5 row [4,...]: 4 at level 2 -> 1; v6 row [5] -> 1.  Total 2."""
+    n, src, dst = _graph(7, [(0, 1), (0, 2), (0, 3), (0, 4), (4, 5), (5, 6)])
+    g = oracle.reorder(oracle.build_csr(n, src, dst))
+    assert g.col[g.row_ptr[0]:g.row_ptr[1]].tolist() == [4, 1, 2, 3]
+    level, _, _ = oracle.bfs(g, 1)
+    assert level.tolist() == [1, 0, 2, 2, 2, 3, 4]
+    assert oracle.bu_probes(g, level, 1) == 6
+    assert oracle.bu_probes(g, level, 2) == 2
+    # k=0 (F_0 = {1}): v0 row [4,1,2,3] hits 1 at index 1 -> 2; v2, v3 -> 1 each (deg);
+    # v4 -> 2; v5 -> 2; v6 -> 1
+    assert oracle.bu_probes(g, level, 0) == 2 + 1 + 1 + 2 + 2 + 1
