@@ -234,14 +234,16 @@ __global__ __launch_bounds__(kExpandThreads, 4) void k_td_expand(KArgs a, int* _
                         }
                     }
                 } else {
-                    // single-scan: the visited bitmap is stale only for this
-                    // level's own discoveries, which just repeat the same level
-                    // value (benign race; any writer's parent is valid, C-26).
-                    const unsigned nx = __ldcg(next + (v >> 5));
-                    if (!((vis | nx) & bit)) {
+                    // single-scan: no status atomics; two threads that both see the
+                    // bit clear write the same level value (benign race; either
+                    // parent is valid, C-26).
+                    // Both bitmaps get fire-and-forget REDs, so later arcs of this
+                    // level mostly see the vertex as visited (one L2 probe per arc).
+                    if (!(vis & bit)) {
                         level[v] = lvl;
                         parent[v] = u;
                         atomicOr(next + (v >> 5), bit);
+                        atomicOr(visited + (v >> 5), bit);
                     }
                 }
             }
@@ -317,7 +319,7 @@ __global__ __launch_bounds__(kGenThreads) void k_generate(KArgs a, int role) {
 // Candidates U_k = not visited (isolated vertices are pre-marked visited).
 // A candidate v is found iff some neighbour is in F_k = fb[k%3] (never a bit set
 // in this same pass: reading C-9), giving level k+1 and that neighbour as parent.
-__global__ __launch_bounds__(kBuThreads) void k_bu_traverse(KArgs a, int* __restrict__ level,
+__global__ __launch_bounds__(kBuThreads, 5) void k_bu_traverse(KArgs a, int* __restrict__ level,
                                                             int* __restrict__ parent) {
     count_launch(a.st);
     const int k = a.st->k;
@@ -357,23 +359,46 @@ __global__ __launch_bounds__(kBuThreads) void k_bu_traverse(KArgs a, int* __rest
         __syncwarp();
         // 2. lane-per-candidate, kBuBatch arcs per step in stored (degree-desc) order;
         //    a lane that finishes takes the next candidate, so lanes stay busy.
+        //    The first probe uses head[v] (deg << 32 | first stored neighbour), a dense
+        //    array read in candidate order; row_ptr/col are touched only on a miss.
         int v = -1, nxt = 0, nhard = 0;
         long long rs = 0, re = 0, p = 0;
+        unsigned long long hd = 0;
+        bool first = false;
         for (;;) {
             const unsigned need = __ballot_sync(FULL, v < 0);
             if (v < 0) {
                 const int idx = nxt + __popc(need & lt);
                 if (idx < total) {
                     v = s_list[wib][idx];
-                    rs = a.row_ptr[v];
-                    re = a.row_ptr[v + 1];
-                    p = rs;
+                    hd = __ldg(a.head + v);
+                    first = true;
                 }
             }
             nxt += __popc(need);
             if (!__any_sync(FULL, v >= 0)) break;
             bool to_hard = false;
-            if (v >= 0) {
+            if (v >= 0 && first) {
+                const int fu = (int)(unsigned)hd;
+                const long long d = (long long)(hd >> 32);
+                if ((__ldcg(cur + (fu >> 5)) >> (fu & 31)) & 1u) {
+                    level[v] = lvl;
+                    parent[v] = fu;
+                    atomicOr(&s_found[wib][(v >> 5) - c * kCW], 1u << (v & 31));
+                    edges += (unsigned long long)d;
+                    ++found;
+                    probes += 1;
+                    v = -1;
+                } else if (d == 1) {
+                    probes += 1;
+                    v = -1;
+                } else {
+                    rs = a.row_ptr[v];
+                    re = rs + d;
+                    p = rs + 1;
+                    first = false;
+                }
+            } else if (v >= 0) {
                 const long long end = min(re, p + kBuBatch);
                 int u[kBuBatch];
                 unsigned wd[kBuBatch];

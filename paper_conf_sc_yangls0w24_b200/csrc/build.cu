@@ -99,6 +99,17 @@ __global__ __launch_bounds__(kB) void k_degree_facts(const long long* __restrict
     }
 }
 
+// head[v] = deg(v) << 32 | first stored neighbour: the bottom-up first probe reads
+// this dense array in candidate order instead of a random sector of col.
+__global__ __launch_bounds__(kB) void k_head(const long long* __restrict__ row_ptr, const int* __restrict__ col,
+                                             long long n, unsigned long long* __restrict__ head) {
+    for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < n;
+         v += (long long)gridDim.x * blockDim.x) {
+        const long long rs = row_ptr[v], d = row_ptr[v + 1] - rs;
+        head[v] = ((unsigned long long)d << 32) | (d > 0 ? (unsigned)col[rs] : 0xffffffffu);
+    }
+}
+
 // Reorder keys: (row << db) | (maxdeg - deg(col))  -> degree descending within the
 // row; the radix sort is stable so ties keep ascending id order (reading C-12).
 // mode 0 keys: (row << nb) | col  -> id order.
@@ -309,6 +320,9 @@ extern "C" xbfs_status xbfs_build_csr(const void* src, const void* dst, int64_t 
     XBFS_CUDA(g, cudaStreamSynchronize(g->stream));
     g->nonisolated_count = (long long)facts[0];
     g->max_deg = (int)facts[1];
+    XBFS_CUDA(g, cudaMalloc(&g->head, n * sizeof(unsigned long long)));
+    k_head<<<grid_for(n), kB, 0, g->stream>>>(g->row_ptr, g->col, n, g->head);
+    XBFS_CUDA(g, cudaGetLastError());
     if ((unsigned long long)arcs >= (1ull << g->dbits))
         return set_error(XBFS_ERR_INVALID_ARG, "graph too large for the packed queue counter");
     guard.keep = true;
@@ -354,6 +368,9 @@ extern "C" xbfs_status xbfs_reorder(xbfs_graph* g, int32_t mode) {
     }
     cudaFree(k0);
     cudaFree(k1);
+    k_head<<<grid_for(n), kB, 0, g->stream>>>(g->row_ptr, g->col, n, g->head);
+    XBFS_CUDA(g, cudaGetLastError());
+    XBFS_CUDA(g, cudaStreamSynchronize(g->stream));
     // the BFS graph (if any) captured the old col pointer
     g->drop_loops();
     g->reorder_mode = mode;

@@ -64,6 +64,7 @@ struct KArgs {
     const int* col;
     int* level;
     int* parent;
+    const unsigned long long* head;  // per vertex: deg << 32 | first stored neighbour (BU first probe)
     unsigned int* visited;
     unsigned int* fb[3];
     int* qv[2];
@@ -94,6 +95,7 @@ struct xbfs_graph {
     int* col = nullptr;
     int* tcount = nullptr;
     unsigned int* nonisolated = nullptr;
+    unsigned long long* head = nullptr;  // deg << 32 | col[row_ptr[v]] (rebuilt by every reorder)
     long long nonisolated_count = 0;
     // BFS work state
     unsigned int* visited = nullptr;
