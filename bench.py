@@ -76,6 +76,20 @@ def pick_roots(cfg_name: str, n, src, dst, count: int):
     return synth.roots(n, src, dst, count, root_seed=ROOT_SEED)
 
 
+def rle(s: str) -> str:
+    """Run-length form of a per-level strategy string (F=SF, S=SS, B=BU) when long."""
+    if len(s) <= 24:
+        return s
+    out, i = [], 0
+    while i < len(s):
+        j = i
+        while j < len(s) and s[j] == s[i]:
+            j += 1
+        out.append(f"{s[i]}{j - i}")
+        i = j
+    return " ".join(out)
+
+
 def load_peaks():
     p = os.path.join(ROOT, "MEASURED_PEAKS.json")
     try:
@@ -202,6 +216,8 @@ def run_ours(args):
         opts["alpha"] = args.alpha
     if args.bu_stay is not None:
         opts["bu_stay"] = args.bu_stay
+    if args.small_edges is not None:
+        opts["small_edges"] = args.small_edges
 
     for r in warm:
         g.run(int(r), level, parent, stats=True, **opts)
@@ -334,7 +350,7 @@ def run_ours(args):
         "kernels": res["kernels"],
         "cpu_baseline": cpu,
         "levels": [pr[4] for pr in res["per_root"][:4]],
-        "strategies": [pr[5] for pr in res["per_root"][:4]],
+        "strategies": [rle(pr[5]) for pr in res["per_root"][:4]],
         "parent_tree_consistent": bool(all(x["ok_tree"] for x in allres)),
         "prep_s": {"generate": round(t_gen, 2), "build_csr": round(t_build, 2), "reorder": round(t_reorder, 2)},
     }
@@ -414,6 +430,7 @@ def main():
     ap.add_argument("--driver", type=int, default=1, help="0 auto, 1 host loop, 2 CUDA-graph device loop")
     ap.add_argument("--alpha", type=float, default=None)
     ap.add_argument("--bu-stay", type=float, default=None)
+    ap.add_argument("--small-edges", type=int, default=None)
     ap.add_argument("--e2e-roots", type=int, default=8)
     ap.add_argument("--profile-roots", type=int, default=4)
     ap.add_argument("--cpu-budget", type=float, default=15.0)

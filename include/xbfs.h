@@ -66,7 +66,8 @@ typedef struct {
     double bu_stay;          /* >0: stay BU while |U_k| * bu_stay < edgesF_k (C-11); default 1.0, 0 = paper rule */
     int32_t force_strategy;  /* -1 adaptive; 0 SF, 1 SS, 2 BU on every level (tests, Fig 7 sweep) */
     int32_t driver;          /* 0 auto, 1 host loop (one sync per level), 2 CUDA-graph device loop */
-    int32_t lazy_init;       /* reserved (0) */
+    int32_t small_edges;     /* SF levels with edgesF_k <= this run inside one thread-block cluster
+                                (small-frontier mode); default 65536, 0 = off, max 73728 */
     int32_t reserved;
 } xbfs_run_opts;
 
@@ -98,7 +99,7 @@ typedef struct {
 
 /* kernel ids reported in xbfs_run_stats.kernel_id */
 enum { XBFS_K_INIT = 0, XBFS_K_SEED = 1, XBFS_K_GENERATE_PRE = 2, XBFS_K_TD_SF = 3, XBFS_K_TD_SS = 4,
-       XBFS_K_GENERATE_POST = 5, XBFS_K_BU = 6, XBFS_K_SELECT = 7 };
+       XBFS_K_GENERATE_POST = 5, XBFS_K_BU = 6, XBFS_K_SELECT = 7, XBFS_K_SMALL = 8 };
 
 /* Fill opts with the defaults (alpha 0.1, grow 2.0, ratio_min 1e-3, bu_stay 1, adaptive). */
 void xbfs_run_opts_default(xbfs_run_opts* opts);

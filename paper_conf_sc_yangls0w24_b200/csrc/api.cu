@@ -39,7 +39,7 @@ xbfs::KArgs xbfs_graph::kargs() const {
     a.visited = visited;
     const long long stride = (words + 31) / 32 * 32;  // 128-byte aligned bitmaps (uint4 access)
     for (int i = 0; i < 3; ++i) a.fb[i] = fb + i * stride;
-    for (int i = 0; i < 2; ++i) {
+    for (int i = 0; i < 3; ++i) {
         a.qv[i] = qv + i * n;
         a.qoff[i] = qoff + i * n;
         a.qdelta[i] = qdelta + i * n;
@@ -75,6 +75,7 @@ void xbfs_run_opts_default(xbfs_run_opts* o) {
     o->ratio_min = 1e-3;  // reading C-10
     o->bu_stay = 1.0;     // reading C-11, tuned on B200 (tools/sweep_selector.py); 0 = paper rule
     o->force_strategy = -1;
+    o->small_edges = 65536;  // small-frontier cluster mode threshold (tuned on the grid config)
     o->driver = 0;
 }
 

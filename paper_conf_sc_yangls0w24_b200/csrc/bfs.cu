@@ -23,9 +23,13 @@
 #include <stdio.h>
 #include <string.h>
 
+#include <cooperative_groups.h>
+
 #include <algorithm>
 
 #include "common.cuh"
+
+namespace cg = cooperative_groups;
 
 namespace xbfs {
 
@@ -47,17 +51,32 @@ __device__ __forceinline__ void clear_stale(const KArgs& a, int k) {
     for (long long i = w4 * 4 + tid; i < a.words; i += nth) z[i] = 0;
 }
 
+// Max-degree tracking without hammering one L2 address: most calls see a value
+// that is already large enough and skip the atomic.
+__device__ __forceinline__ void atomic_max_if_greater(unsigned* p, unsigned v) {
+    if (v > __ldcg(p)) atomicMax(p, v);
+}
+
+// Warp-reduce a per-lane max and publish it (call with the whole warp converged).
+__device__ __forceinline__ void flush_max(unsigned* p, unsigned lmax) {
+    const unsigned w = __reduce_max_sync(FULL, lmax);
+    if ((threadIdx.x & 31) == 0 && w) atomic_max_if_greater(p, w);
+}
+
 // Warp-aggregated enqueue of the lanes with `win` set: one 64-bit atomicAdd on
 // the packed counter returns both the queue slot base (high bits) and the degree
 // offset base (low dbits), so qoff is an exact exclusive prefix sum of degrees
 // over the queue, in slot order.  Every tile start (multiple of kTile) that falls
 // inside a vertex's arc range records that vertex's slot in tile_first.
+// lmax accumulates the lane's max enqueued degree; the kernel publishes it once
+// at the end with flush_max (no extra round trip inside the hot loop).
 __device__ __forceinline__ void enqueue_warp(bool win, int v, long long rs, long long deg,
-                                             unsigned long long* ctr, int dbits, int* qv, long long* qoff,
-                                             long long* qdelta, int* tile_first) {
+                                             unsigned long long* ctr, unsigned& lmax, int dbits, int* qv,
+                                             long long* qoff, long long* qdelta, int* tile_first) {
     const unsigned mask = __ballot_sync(FULL, win);
     if (mask == 0) return;
     const int lane = threadIdx.x & 31;
+    if (win) lmax = max(lmax, (unsigned)deg);
     const int rank = __popc(mask & ((1u << lane) - 1u));
     long long d = win ? deg : 0;
     long long incl = d;
@@ -82,6 +101,65 @@ __device__ __forceinline__ void enqueue_warp(bool win, int v, long long rs, long
             for (long long t = t0; t <= t1; ++t) tile_first[t] = (int)slot;
         }
     }
+}
+
+// Same as enqueue_warp for up to R winners per lane (one atomic per warp).
+template <int R>
+__device__ __forceinline__ void enqueue_warp_multi(const bool (&win)[R], const int (&v)[R], const long long (&rs)[R],
+                                                   const long long (&deg)[R], unsigned long long* ctr, unsigned& lmax,
+                                                   int dbits, int* qv, long long* qoff, long long* qdelta,
+                                                   int* tile_first) {
+    int cnt = 0;
+    long long dsum = 0;
+#pragma unroll
+    for (int i = 0; i < R; ++i)
+        if (win[i]) { ++cnt; dsum += deg[i]; lmax = max(lmax, (unsigned)deg[i]); }
+    if (!__any_sync(FULL, cnt > 0)) return;
+    const int lane = threadIdx.x & 31;
+    int ic = cnt;
+    long long id = dsum;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const int tc = __shfl_up_sync(FULL, ic, o);
+        const long long td = __shfl_up_sync(FULL, id, o);
+        if (lane >= o) { ic += tc; id += td; }
+    }
+    const int wc = __shfl_sync(FULL, ic, 31);
+    const long long wd = __shfl_sync(FULL, id, 31);
+    unsigned long long base = 0;
+    if (lane == 0) base = atomicAdd(ctr, ((unsigned long long)wc << dbits) + (unsigned long long)wd);
+    base = __shfl_sync(FULL, base, 0);
+    long long slot = (long long)(base >> dbits) + ic - cnt;
+    long long off = (long long)(base & ((1ull << dbits) - 1ull)) + id - dsum;
+#pragma unroll
+    for (int i = 0; i < R; ++i) {
+        if (!win[i]) continue;
+        qv[slot] = v[i];
+        qoff[slot] = off;
+        qdelta[slot] = rs[i] - off;
+        if (deg[i] > 0) {
+            const long long t0 = (off + kTile - 1) / kTile, t1 = (off + deg[i] - 1) / kTile;
+            for (long long t = t0; t <= t1; ++t) tile_first[t] = (int)slot;
+        }
+        ++slot;
+        off += deg[i];
+    }
+}
+
+// The host-loop driver reads the level state from pinned, mapped host memory:
+// one 32-byte store per level (skipped by the CUDA-graph driver).
+__device__ __forceinline__ void mirror_host(const KArgs& a, const DevState* st) {
+    if (!st->mirror_host) return;
+    HostCtl h;
+    h.k = st->k;
+    h.strategy = st->strategy;
+    h.queue_valid = st->queue_valid;
+    h.done = st->done;
+    h.fsize = st->fsize;
+    h.fedges = st->fedges;
+    h.fmaxdeg = st->fmaxdeg;
+    h.prev_small = st->prev_small;
+    *a.hctl = h;
 }
 
 // ---------------------------------------------------------------- init
@@ -140,6 +218,12 @@ __global__ void k_seed(KArgs a, int* level, int* parent, long long nonisolated_c
     st->k = 0;
     st->qctr[0] = (1ull << a.dbits) + (unsigned long long)deg;
     st->qctr[1] = 0;
+    st->qctr[2] = 0;
+    st->qmax[0] = (unsigned)deg;
+    st->qmax[1] = 0;
+    st->qmax[2] = 0;
+    st->fmaxdeg = (unsigned)deg;
+    st->prev_small = 0;
     st->queue_valid = 1;
     st->done = 0;
     st->fsize = 1;
@@ -153,10 +237,7 @@ __global__ void k_seed(KArgs a, int* level, int* parent, long long nonisolated_c
     st->source = s;
     st->prev_strategy = -1;
     st->strategy = choose_strategy(st, a.arcs, 1, 0, deg, st->unvisited, -1);
-    a.hctl->k = 0;
-    a.hctl->strategy = st->strategy;
-    a.hctl->queue_valid = 1;
-    a.hctl->done = 0;
+    mirror_host(a, st);
 }
 
 // ----------------------------------------------------------- top-down
@@ -165,13 +246,13 @@ __global__ void k_seed(KArgs a, int* level, int* parent, long long nonisolated_c
 // (hubs span many tiles, small vertices share one).  Arc a of the frontier is
 // col[a + qdelta[j]] for its owner j (binary search of qoff in shared memory).
 template <int MODE>
-__global__ __launch_bounds__(kExpandThreads, 4) void k_td_expand(KArgs a, int* __restrict__ level,
+__global__ __launch_bounds__(kExpandThreads, 3) void k_td_expand(KArgs a, int* __restrict__ level,
                                                                 int* __restrict__ parent) {
     count_launch(a.st);
     const int k = a.st->k;
     clear_stale(a, k);
-    const int in = k & 1, ob = (k + 1) & 1;
-    const unsigned long long q = a.st->qctr[in];
+    const int in = k % 3, ob = (k + 1) % 3;
+    const unsigned long long q = a.st->qctr[k % 3];
     const long long F = (long long)(q >> a.dbits);
     const long long T = (long long)(q & ((1ull << a.dbits) - 1ull));
     if (F == 0 || T == 0) return;
@@ -187,6 +268,7 @@ __global__ __launch_bounds__(kExpandThreads, 4) void k_td_expand(KArgs a, int* _
     __shared__ long long s_off[kTile + 1];
     __shared__ long long s_delta[kTile + 1];
     __shared__ int s_v[kTile + 1];
+    unsigned lmax = 0;
 
     for (long long t = blockIdx.x; t < ntiles; t += gridDim.x) {
         const long long a0 = t * kTile;
@@ -201,57 +283,75 @@ __global__ __launch_bounds__(kExpandThreads, 4) void k_td_expand(KArgs a, int* _
             s_v[i] = qv[i0 + i];
         }
         __syncthreads();
-        int j = 0;
-#pragma unroll 1
-        for (int it = 0; it < kTile / kExpandThreads; ++it) {
-            const long long arc = a0 + it * kExpandThreads + threadIdx.x;
-            const bool valid = arc < a1;
-            bool win = false;
-            int v = 0;
-            long long rs = 0, deg = 0;
-            if (valid) {
-                // owner: last j with s_off[j] <= arc (arcs of a thread increase)
-                int lo = j, hi = nv - 1;
+        // R arcs per thread (stride blockDim: coalesced col reads), processed
+        // stage by stage so the R dependent load chains are in flight together.
+        constexpr int R = kTile / kExpandThreads;
+        int v[R], u[R];
+        unsigned vis[R];
+        bool valid[R], win[R];
+        long long rs[R], deg[R];
+#pragma unroll
+        for (int i = 0; i < R; ++i) {
+            const long long arc = a0 + i * kExpandThreads + threadIdx.x;
+            valid[i] = arc < a1;
+            v[i] = 0;
+            u[i] = 0;
+            if (valid[i]) {
+                // owner: last j with s_off[j] <= arc
+                int lo = 0, hi = nv - 1;
                 while (lo < hi) {
                     const int mid = (lo + hi + 1) >> 1;
                     if (s_off[mid] <= arc) lo = mid; else hi = mid - 1;
                 }
-                j = lo;
-                v = __ldg(a.col + arc + s_delta[j]);
-                const int u = s_v[j];
-                const unsigned bit = 1u << (v & 31);
-                const unsigned vis = __ldcg(visited + (v >> 5));
-                if (MODE == XBFS_SF) {
-                    if (!(vis & bit)) {
-                        const unsigned old = atomicOr(visited + (v >> 5), bit);
-                        if (!(old & bit)) {
-                            win = true;
-                            level[v] = lvl;
-                            parent[v] = u;
-                            atomicOr(next + (v >> 5), bit);
-                            rs = a.row_ptr[v];
-                            deg = a.row_ptr[v + 1] - rs;
-                        }
-                    }
-                } else {
-                    // single-scan: no status atomics; two threads that both see the
-                    // bit clear write the same level value (benign race; either
-                    // parent is valid, C-26).
-                    // Both bitmaps get fire-and-forget REDs, so later arcs of this
-                    // level mostly see the vertex as visited (one L2 probe per arc).
-                    if (!(vis & bit)) {
-                        level[v] = lvl;
-                        parent[v] = u;
-                        atomicOr(next + (v >> 5), bit);
-                        atomicOr(visited + (v >> 5), bit);
-                    }
+                v[i] = __ldg(a.col + arc + s_delta[lo]);
+                u[i] = s_v[lo];
+            }
+        }
+#pragma unroll
+        for (int i = 0; i < R; ++i) vis[i] = valid[i] ? __ldcg(visited + (v[i] >> 5)) : FULL;
+        if (MODE == XBFS_SF) {
+            unsigned old[R];
+#pragma unroll
+            for (int i = 0; i < R; ++i) {
+                const unsigned bit = 1u << (v[i] & 31);
+                old[i] = (vis[i] & bit) ? bit : atomicOr(visited + (v[i] >> 5), bit);
+            }
+#pragma unroll
+            for (int i = 0; i < R; ++i) {
+                const unsigned bit = 1u << (v[i] & 31);
+                win[i] = valid[i] && !(old[i] & bit);
+                rs[i] = 0;
+                deg[i] = 0;
+                if (win[i]) {
+                    level[v[i]] = lvl;
+                    parent[v[i]] = u[i];
+                    atomicOr(next + (v[i] >> 5), bit);
+                    rs[i] = a.row_ptr[v[i]];
+                    deg[i] = a.row_ptr[v[i] + 1];
                 }
             }
-            if (MODE == XBFS_SF)
-                enqueue_warp(win, v, rs, deg, &a.st->qctr[ob], a.dbits, a.qv[ob], a.qoff[ob], a.qdelta[ob],
-                             a.tile_first[ob]);
+#pragma unroll
+            for (int i = 0; i < R; ++i) deg[i] -= rs[i];
+            enqueue_warp_multi<R>(win, v, rs, deg, &a.st->qctr[(k + 1) % 3], lmax, a.dbits, a.qv[ob],
+                                  a.qoff[ob], a.qdelta[ob], a.tile_first[ob]);
+        } else {
+            // single-scan: no status atomics; two threads that both see the bit
+            // clear write the same level value (benign race; either parent is
+            // valid, C-26).  Both bitmaps get fire-and-forget REDs, so later arcs
+            // of this level mostly see the vertex as visited (one probe per arc).
+#pragma unroll
+            for (int i = 0; i < R; ++i) {
+                const unsigned bit = 1u << (v[i] & 31);
+                if (valid[i] && !(vis[i] & bit)) {
+                    level[v[i]] = lvl;
+                    parent[v[i]] = u[i];
+                    atomicOr(next + (v[i] >> 5), bit);
+                    atomicOr(visited + (v[i] >> 5), bit);
+                }
+            }
         }
     }
+    if (MODE == XBFS_SF) flush_max(&a.st->qmax[(k + 1) % 3], lmax);
 }
 
 // -------------------------------------------------------------- generate
@@ -263,11 +363,12 @@ __global__ __launch_bounds__(kGenThreads) void k_generate(KArgs a, int role) {
     count_launch(a.st);
     const int k = a.st->k;
     const unsigned int* __restrict__ bm = role == 0 ? a.fb[k % 3] : a.fb[(k + 1) % 3];
-    const int ob = role == 0 ? (k & 1) : ((k + 1) & 1);
-    unsigned long long* ctr = &a.st->qctr[ob];
+    const int ob = role == 0 ? k % 3 : (k + 1) % 3;
+    unsigned long long* ctr = &a.st->qctr[role == 0 ? k % 3 : (k + 1) % 3];
     const long long nth = (long long)gridDim.x * blockDim.x;
     const long long base_tid = blockIdx.x * (long long)blockDim.x + (threadIdx.x & ~31);
     const int lane = threadIdx.x & 31;
+    unsigned gmax = 0;
     for (long long w0 = base_tid; w0 < a.words; w0 += nth) {
         const long long w = w0 + lane;
         unsigned word = w < a.words ? bm[w] : 0u;
@@ -277,7 +378,9 @@ __global__ __launch_bounds__(kGenThreads) void k_generate(KArgs a, int role) {
         long long dsum = 0;
         for (unsigned b = word; b; b &= b - 1) {
             const long long v = w * 32 + __ffs(b) - 1;
-            dsum += a.row_ptr[v + 1] - a.row_ptr[v];
+            const long long d = a.row_ptr[v + 1] - a.row_ptr[v];
+            dsum += d;
+            gmax = max(gmax, (unsigned)d);
         }
         int ic = cnt;
         long long id = dsum;
@@ -313,6 +416,7 @@ __global__ __launch_bounds__(kGenThreads) void k_generate(KArgs a, int role) {
             off += deg;
         }
     }
+    flush_max(&a.st->qmax[role == 0 ? k % 3 : (k + 1) % 3], gmax);
 }
 
 // ------------------------------------------------------------- bottom-up
@@ -338,6 +442,7 @@ __global__ __launch_bounds__(kBuThreads, 5) void k_bu_traverse(KArgs a, int* __r
     const long long gw = (blockIdx.x * (long long)blockDim.x + threadIdx.x) >> 5;
     const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
     unsigned long long found = 0, edges = 0, probes = 0;
+    unsigned fmax = 0;
     for (long long c = gw; c < nchunks; c += nw) {
         // 1. candidates of kCW bitmap words: ballot/popc compaction into shared memory
         //    (the paper's count + prefix-sum + queue-write "double scan").
@@ -386,6 +491,7 @@ __global__ __launch_bounds__(kBuThreads, 5) void k_bu_traverse(KArgs a, int* __r
                     parent[v] = fu;
                     atomicOr(&s_found[wib][(v >> 5) - c * kCW], 1u << (v & 31));
                     edges += (unsigned long long)d;
+                    fmax = max(fmax, (unsigned)d);
                     ++found;
                     probes += 1;
                     v = -1;
@@ -418,6 +524,7 @@ __global__ __launch_bounds__(kBuThreads, 5) void k_bu_traverse(KArgs a, int* __r
                     parent[v] = pu;
                     atomicOr(&s_found[wib][(v >> 5) - c * kCW], 1u << (v & 31));
                     edges += (unsigned long long)(re - rs);
+                    fmax = max(fmax, (unsigned)(re - rs));
                     ++found;
                     probes += (unsigned long long)(p + hit + 1 - rs);
                     v = -1;
@@ -457,6 +564,7 @@ __global__ __launch_bounds__(kBuThreads, 5) void k_bu_traverse(KArgs a, int* __r
                         parent[hv] = u;
                         atomicOr(&s_found[wib][(hv >> 5) - c * kCW], 1u << (hv & 31));
                         edges += (unsigned long long)(hre - hrs);
+                        fmax = max(fmax, (unsigned)(hre - hrs));
                         ++found;
                         probes += (unsigned long long)(pp + 1 - hrs);
                     }
@@ -485,6 +593,10 @@ __global__ __launch_bounds__(kBuThreads, 5) void k_bu_traverse(KArgs a, int* __r
         atomicAdd(&a.st->acc_edges, edges);
         atomicAdd(&a.st->acc_probes, probes);
     }
+    fmax = __reduce_max_sync(FULL, fmax);
+    if (lane == 0 && fmax) {
+        atomic_max_if_greater(&a.st->qmax[(k + 1) % 3], fmax);
+    }
 }
 
 // ---------------------------------------------------------------- select
@@ -492,6 +604,11 @@ template <bool kGraph>
 __global__ void k_select(KArgs a, cudaGraphConditionalHandle h_while) {
     count_launch(a.st);
     DevState* st = a.st;
+    if (st->advanced) {             // k_small already ran its levels and advanced the state
+        st->advanced = 0;
+        if (kGraph) cudaGraphSetConditional(h_while, st->done ? 0u : 1u);
+        return;
+    }
     const int k = st->k;
     const int strat = st->strategy;
     long long nf, ne;
@@ -500,7 +617,7 @@ __global__ void k_select(KArgs a, cudaGraphConditionalHandle h_while) {
         ne = (long long)st->acc_edges;
         st->queue_valid = 0;
     } else {
-        const unsigned long long q = st->qctr[(k + 1) & 1];
+        const unsigned long long q = st->qctr[(k + 1) % 3];
         nf = (long long)(q >> a.dbits);
         ne = (long long)(q & ((1ull << a.dbits) - 1ull));
         st->queue_valid = 1;
@@ -515,6 +632,9 @@ __global__ void k_select(KArgs a, cudaGraphConditionalHandle h_while) {
         r.pad = 0;
         a.log[k] = r;
     }
+    // enter the small-frontier mode only after one small SF level has already run
+    // through the level kernels (a single small level does not pay for the switch)
+    st->prev_small = strat == XBFS_SF && st->fedges <= st->small_edges && st->fmaxdeg <= (unsigned)kSmallMaxDeg;
     st->reached += st->fsize;
     st->arcs_traversed += st->fedges;
     st->fprev = st->fsize;
@@ -524,27 +644,208 @@ __global__ void k_select(KArgs a, cudaGraphConditionalHandle h_while) {
     st->acc_found = st->acc_edges = st->acc_probes = 0;
     st->prev_strategy = strat;
     st->k = k + 1;
+    st->fmaxdeg = st->qmax[(k + 1) % 3];
+    st->qctr[(k + 2) % 3] = 0;   // counter of the queue built during level k+1
+    st->qmax[(k + 2) % 3] = 0;
     if (nf == 0) {
         st->done = 1;
         st->nlevels = k + 1;
     } else {
         st->strategy = choose_strategy(st, a.arcs, nf, st->fprev, ne, st->unvisited, strat);
-        st->qctr[(k + 2) & 1] = 0;                   // queue buffer built during level k+1
-        if (!st->queue_valid) st->qctr[(k + 1) & 1] = 0;  // rebuilt by generate(role 0)
     }
-    a.hctl->k = st->k;
-    a.hctl->strategy = st->strategy;
-    a.hctl->queue_valid = st->queue_valid;
-    a.hctl->done = st->done;
+    mirror_host(a, st);
     if (kGraph) cudaGraphSetConditional(h_while, st->done ? 0u : 1u);
+}
+
+// Small-frontier cluster mode gate: a scan-free level whose frontier has at most
+// small_edges arcs and no vertex above kSmallMaxDeg (a hub would serialise a warp).
+__host__ __device__ __forceinline__ bool small_gate(long long small_edges, int strategy, int queue_valid,
+                                                    long long fedges, unsigned maxdeg) {
+    return strategy == XBFS_SF && queue_valid && fedges <= small_edges && maxdeg <= (unsigned)kSmallMaxDeg;
+}
+
+__device__ __forceinline__ bool small_mode(const DevState* st, int strategy, int queue_valid, long long fedges,
+                                           unsigned maxdeg) {
+    return small_gate(st->small_edges, strategy, queue_valid, fedges, maxdeg);
 }
 
 // Device loop: map (strategy, queue_valid) of level k to a SWITCH branch.
 __global__ void k_plan(KArgs a, cudaGraphConditionalHandle h_switch) {
     count_launch(a.st);
     const int s = a.st->strategy, qv = a.st->queue_valid;
-    const unsigned br = s == XBFS_BU ? 4u : (s == XBFS_SF ? (qv ? 0u : 1u) : (qv ? 2u : 3u));
+    unsigned br = s == XBFS_BU ? 4u : (s == XBFS_SF ? (qv ? 0u : 1u) : (qv ? 2u : 3u));
+    if (a.st->prev_small && small_mode(a.st, s, qv, a.st->fedges, a.st->fmaxdeg)) br = 5u;
     cudaGraphSetConditional(h_switch, br);
+}
+
+// --------------------------------------------------- small-frontier mode
+// One thread-block cluster (kSmallCluster CTAs x 1024 threads) runs consecutive
+// scan-free levels while edgesF_k <= small_edges: the level
+// barrier is a cluster barrier (~hundreds of ns) instead of a kernel boundary +
+// host round trip, which is what bounds the many tiny levels of a grid graph
+// (small/many-level graphs are dominated by CPU-GPU interaction).
+// Vertex-per-thread for deg <= kSmallInline (all arcs' loads in flight at once),
+// warp-per-vertex (32 arcs per step) for the rest.  The frontier bitmaps keep the
+// level kernels' invariant exactly but cheaply: winners RED their bit into
+// fb[(k+1)%3], and the stale F_{k-1} bits are unset one by one from its queue
+// (buffer (k+2)%3, untouched during level k) instead of clearing N/8 bytes.
+__device__ __forceinline__ bool sf_claim(unsigned int* visited, int v) {
+    const unsigned bit = 1u << (v & 31);
+    if (__ldcg(visited + (v >> 5)) & bit) return false;
+    return !(atomicOr(visited + (v >> 5), bit) & bit);
+}
+
+__global__ void __cluster_dims__(kSmallCluster, 1, 1) __launch_bounds__(kSmallThreads, 1) k_small_sf(KArgs a, int* __restrict__ level,
+                                                             int* __restrict__ parent) {
+    count_launch(a.st);
+    cg::cluster_group cl = cg::this_cluster();
+    const int crank = (int)cl.block_rank(), csize = (int)cl.num_blocks();
+    DevState* st = a.st;
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
+    __shared__ int s_big[kSmallBig];
+    __shared__ int s_nbig;
+    int k = st->k;
+    long long fsize = st->fsize, fedges = st->fedges, fprev = st->fprev, unvisited = st->unvisited;
+    long long reached = st->reached, arcs_tr = st->arcs_traversed;
+    unsigned fmaxdeg = st->fmaxdeg;
+    bool done = false;
+    int next_strat = XBFS_SF;
+    const long long tid = (long long)crank * blockDim.x + threadIdx.x;
+    const long long nth = (long long)csize * blockDim.x;
+    cl.sync();                      // every CTA has read the state before CTA 0 touches it
+    for (;;) {
+        const int in = k % 3, ob = (k + 1) % 3;
+        unsigned long long* octr = &st->qctr[(k + 1) % 3];
+        unsigned* omax = &st->qmax[(k + 1) % 3];
+        unsigned lmax = 0;
+        unsigned int* next = a.fb[(k + 1) % 3];
+        if (crank == 0 && threadIdx.x == 0) {
+            st->qctr[(k + 2) % 3] = 0;
+            st->qmax[(k + 2) % 3] = 0;
+        }
+        if (threadIdx.x == 0) s_nbig = 0;
+        {   // unset the stale F_{k-1} bits (its queue is buffer (k+2)%3)
+            unsigned int* stale = a.fb[(k + 2) % 3];
+            const int* pq = a.qv[(k + 2) % 3];
+            for (long long j = tid; j < fprev; j += nth) {
+                const int v = pq[j];
+                atomicAnd(stale + (v >> 5), ~(1u << (v & 31)));
+            }
+        }
+        __syncthreads();
+        const int* qv = a.qv[in];
+        const long long* qoff = a.qoff[in];
+        const long long* qdelta = a.qdelta[in];
+        const int lvl = k + 1;
+        const long long rounds = (fsize + nth - 1) / nth;
+        for (long long r = 0; r < rounds; ++r) {
+            const long long j = r * nth + tid;
+            int u = 0;
+            long long rs = 0, d = 0;
+            if (j < fsize) {
+                u = qv[j];
+                const long long o = qoff[j];
+                rs = o + qdelta[j];
+                d = (j + 1 < fsize ? qoff[j + 1] : fedges) - o;
+                if (d > kSmallInline) {
+                    s_big[atomicAdd(&s_nbig, 1)] = (int)j;   // cannot overflow: small_edges <= 9*kSmallBig
+                    d = 0;
+                }
+            }
+            int v[kSmallInline];
+            bool win[kSmallInline];
+            long long vrs[kSmallInline], vdeg[kSmallInline];
+#pragma unroll
+            for (int i = 0; i < kSmallInline; ++i) v[i] = i < d ? __ldg(a.col + rs + i) : -1;
+#pragma unroll
+            for (int i = 0; i < kSmallInline; ++i) {
+                win[i] = v[i] >= 0 && sf_claim(a.visited, v[i]);
+                vrs[i] = 0;
+                vdeg[i] = 0;
+                if (win[i]) {
+                    level[v[i]] = lvl;
+                    parent[v[i]] = u;
+                    atomicOr(next + (v[i] >> 5), 1u << (v[i] & 31));
+                    vrs[i] = a.row_ptr[v[i]];
+                    vdeg[i] = a.row_ptr[v[i] + 1];
+                }
+            }
+#pragma unroll
+            for (int i = 0; i < kSmallInline; ++i) vdeg[i] -= vrs[i];
+            enqueue_warp_multi<kSmallInline>(win, v, vrs, vdeg, octr, lmax, a.dbits, a.qv[ob], a.qoff[ob], a.qdelta[ob],
+                                             a.tile_first[ob]);
+        }
+        __syncthreads();
+        const int nbig = s_nbig;
+        for (int b = wid; b < nbig; b += nwarps) {
+            const long long j = s_big[b];
+            const int bu = qv[j];
+            const long long o = qoff[j];
+            const long long rs = o + qdelta[j];
+            const long long d = (j + 1 < fsize ? qoff[j + 1] : fedges) - o;
+            for (long long base = 0; base < d; base += 32) {
+                const long long p = base + lane;
+                const int v = p < d ? __ldg(a.col + rs + p) : -1;
+                const bool w = v >= 0 && sf_claim(a.visited, v);
+                long long vrs = 0, vdeg = 0;
+                if (w) {
+                    level[v] = lvl;
+                    parent[v] = bu;
+                    atomicOr(next + (v >> 5), 1u << (v & 31));
+                    vrs = a.row_ptr[v];
+                    vdeg = a.row_ptr[v + 1] - vrs;
+                }
+                enqueue_warp(w, v, vrs, vdeg, octr, lmax, a.dbits, a.qv[ob], a.qoff[ob], a.qdelta[ob],
+                             a.tile_first[ob]);
+            }
+        }
+        flush_max(omax, lmax);
+        cl.sync();                  // level barrier: all claims and enqueues of level k are visible
+        const unsigned long long q = atomicAdd(octr, 0ull);
+        const unsigned nmax = atomicOr(omax, 0u);
+        const long long nf = (long long)(q >> a.dbits);
+        const long long ne = (long long)(q & ((1ull << a.dbits) - 1ull));
+        if (crank == 0 && threadIdx.x == 0 && k < kLogCap) {
+            LevelRec rec;
+            rec.fsize = fsize;
+            rec.fedges = fedges;
+            rec.unvisited = unvisited;
+            rec.probes = 0;
+            rec.strategy = XBFS_SF;
+            rec.pad = 0;
+            a.log[k] = rec;
+        }
+        reached += fsize;
+        arcs_tr += fedges;
+        fprev = fsize;
+        unvisited -= nf;
+        fsize = nf;
+        fedges = ne;
+        fmaxdeg = nmax;
+        ++k;
+        if (nf == 0) { done = true; break; }
+        next_strat = choose_strategy(st, a.arcs, nf, fprev, ne, unvisited, XBFS_SF);
+        if (!small_mode(st, next_strat, 1, ne, nmax)) break;
+    }
+    if (crank == 0 && threadIdx.x == 0) {
+        st->k = k;
+        st->strategy = next_strat;
+        st->queue_valid = 1;
+        st->done = done ? 1 : 0;
+        if (done) st->nlevels = k;
+        st->fsize = fsize;
+        st->fedges = fedges;
+        st->fprev = fprev;
+        st->unvisited = unvisited;
+        st->reached = reached;
+        st->arcs_traversed = arcs_tr;
+        st->prev_strategy = XBFS_SF;
+        st->acc_found = st->acc_edges = st->acc_probes = 0;
+        st->fmaxdeg = fmaxdeg;
+        st->advanced = 1;
+        st->prev_small = 1;
+        mirror_host(a, st);
+    }
 }
 
 // Graph500 m (O-6) = sum of tuple counts over reached vertices; untimed.
@@ -565,12 +866,35 @@ struct Grids {
     int init, expand, gen, bu;
 };
 
+// One wave of resident blocks per kernel (grid-stride loops inside), sized from
+// the occupancy calculator once per device.
 Grids grids_for(const xbfs_graph* g) {
+    static int occ[4] = {0, 0, 0, 0};
+    if (!occ[0]) {
+        int o = 0;
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, k_init_fill, 256, 0);
+        occ[0] = std::max(o, 1);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, k_td_expand<XBFS_SF>, kExpandThreads, 0);
+        occ[1] = std::max(o, 1);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, k_generate, kGenThreads, 0);
+        occ[2] = std::max(o, 1);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, k_bu_traverse, kBuThreads, 0);
+        occ[3] = std::max(o, 1);
+    }
+    // XBFS_GRID_{EXPAND,GEN,BU}: blocks per SM override (tuning experiments only)
+    static int ov[3] = {-1, -1, -1};
+    if (ov[0] < 0) {
+        const char* names[3] = {"XBFS_GRID_EXPAND", "XBFS_GRID_GEN", "XBFS_GRID_BU"};
+        for (int i = 0; i < 3; ++i) {
+            const char* e = getenv(names[i]);
+            ov[i] = e ? atoi(e) : 0;
+        }
+    }
     Grids r;
-    r.init = g->num_sms * 8;
-    r.expand = g->num_sms * 4;   // 4 x 512 threads resident per SM
-    r.gen = g->num_sms * 8;
-    r.bu = g->num_sms * 8;       // 8 x 256 threads resident per SM
+    r.init = g->num_sms * std::max(occ[0], 8);   // streaming fill: as many threads as fit
+    r.expand = g->num_sms * (ov[0] > 0 ? ov[0] : occ[1]);
+    r.gen = g->num_sms * (ov[1] > 0 ? ov[1] : occ[2]);
+    r.bu = g->num_sms * (ov[2] > 0 ? ov[2] : occ[3]);
     return r;
 }
 
@@ -627,9 +951,15 @@ struct Prof {
 
 // Enqueue one level given the host-known strategy / queue state.
 xbfs_status launch_level(xbfs_graph* g, const KArgs& a, int* level, int* parent, int k, int strat,
-                         int queue_valid, Prof& P) {
+                         int queue_valid, long long fedges, unsigned maxdeg, int prev_small, long long small_edges,
+                         Prof& P) {
     const Grids G = grids_for(g);
     cudaStream_t s = g->stream;
+    if (prev_small && small_gate(small_edges, strat, queue_valid, fedges, maxdeg)) {
+        XBFS_LAUNCH(P, XBFS_K_SMALL, k, (k_small_sf<<<kSmallCluster, kSmallThreads, 0, s>>>(a, level, parent)));
+        XBFS_LAUNCH(P, XBFS_K_SELECT, k, (k_select<false><<<1, 1, 0, s>>>(a, 0)));
+        return XBFS_OK;
+    }
     if (strat != XBFS_BU && !queue_valid)
         XBFS_LAUNCH(P, XBFS_K_GENERATE_PRE, k, (k_generate<<<G.gen, kGenThreads, 0, s>>>(a, 0)));
     if (strat == XBFS_SF) {
@@ -646,14 +976,17 @@ xbfs_status launch_level(xbfs_graph* g, const KArgs& a, int* level, int* parent,
     return XBFS_OK;
 }
 
-xbfs_status run_host_loop(xbfs_graph* g, const KArgs& a, int* level, int* parent, Prof& P) {
+xbfs_status run_host_loop(xbfs_graph* g, const KArgs& a, int* level, int* parent, long long small_edges,
+                          Prof& P) {
     // k_seed wrote hctl; wait for it, then one sync per level (P:L151's
     // host/device crossing, kept as the debug / measurement driver).
     XBFS_CUDA(g, cudaStreamSynchronize(g->stream));
     for (;;) {
         volatile HostCtl* h = g->hctl;
         if (h->done) break;
-        XBFS_TRY(launch_level(g, a, level, parent, h->k, h->strategy, h->queue_valid, P));
+        XBFS_TRY(launch_level(g, a, level, parent, h->k, h->strategy, h->queue_valid, h->fedges, h->fmaxdeg,
+                              h->prev_small,
+                              small_edges, P));
         XBFS_CUDA(g, cudaStreamSynchronize(g->stream));
     }
     return XBFS_OK;
@@ -722,7 +1055,7 @@ xbfs_status build_loop_graph(xbfs_graph* g, int* level, int* parent) {
     sp.type = cudaGraphNodeTypeConditional;
     sp.conditional.handle = h_switch;
     sp.conditional.type = cudaGraphCondTypeSwitch;
-    sp.conditional.size = 5;
+    sp.conditional.size = 6;
     XBFS_CUDA(g, cudaGraphAddNode(&n_sw, body, &n_plan, 1, &sp));
     cudaGraph_t* br = sp.conditional.phGraph_out;
     int role0 = 0, role1 = 1;
@@ -746,6 +1079,8 @@ xbfs_status build_loop_graph(xbfs_graph* g, int* level, int* parent) {
     XBFS_TRY(add_kernel(g, br[3], &x, &y, f_gen, G.gen, kGenThreads, a_gen1));
     // 4: BU
     XBFS_TRY(add_kernel(g, br[4], &x, nullptr, (void*)k_bu_traverse, G.bu, kBuThreads, a_exp));
+    // 5: small-frontier cluster mode (cluster dims are compiled into the kernel)
+    XBFS_TRY(add_kernel(g, br[5], &x, nullptr, (void*)k_small_sf, kSmallCluster, kSmallThreads, a_exp));
     {
         void* args[] = {&a, &h_while};
         XBFS_TRY(add_kernel(g, body, &n_sel, &n_sw, (void*)k_select<true>, 1, 1, args));
@@ -778,6 +1113,7 @@ static xbfs_status run_impl(xbfs_graph* g, int64_t source, int32_t* level, int32
     XBFS_CUDA(g, cudaSetDevice(g->device));
 
     KArgs a = g->kargs();
+    const bool use_graph = (o.driver == 0 || o.driver == 2) && !(stats && stats->kernel_capacity > 0);
     // selection parameters live in the device state
     {
         DevState hs;
@@ -788,13 +1124,14 @@ static xbfs_status run_impl(xbfs_graph* g, int64_t source, int32_t* level, int32
         hs.bu_stay = o.bu_stay;
         hs.force = o.force_strategy;
         hs.source = source;
+        hs.small_edges = std::min<long long>(std::max(o.small_edges, 0), kSmallEdgesMax);
+        hs.mirror_host = use_graph ? 0 : 1;
         XBFS_CUDA(g, cudaMemcpyAsync(g->st, &hs, sizeof(hs), cudaMemcpyHostToDevice, g->stream));
     }
     const Grids G = grids_for(g);
     Prof P;
     P.g = g;
     P.st = stats;
-    const bool use_graph = (o.driver == 0 || o.driver == 2) && !(stats && stats->kernel_capacity > 0);
     if (use_graph) {
         XBFS_TRY(build_loop_graph(g, level, parent));
         XBFS_CUDA(g, cudaEventRecord(g->ev0, g->stream));
@@ -806,7 +1143,7 @@ static xbfs_status run_impl(xbfs_graph* g, int64_t source, int32_t* level, int32
                 (k_init_fill<<<G.init, 256, 0, g->stream>>>(a, level, parent, g->nonisolated)));
     XBFS_LAUNCH(P, XBFS_K_SEED, -1,
                 (k_seed<<<1, 1, 0, g->stream>>>(a, level, parent, g->nonisolated_count)));
-    XBFS_TRY(run_host_loop(g, a, level, parent, P));
+    XBFS_TRY(run_host_loop(g, a, level, parent, std::min<long long>(std::max(o.small_edges, 0), kSmallEdgesMax), P));
     XBFS_CUDA(g, cudaEventRecord(g->ev1, g->stream));
     }
 

@@ -171,10 +171,10 @@ xbfs_status alloc_work(xbfs_graph* g) {
     g->tiles_cap = g->arcs / kTile + 4;
     XBFS_CUDA(g, cudaMalloc(&g->visited, words * sizeof(unsigned int)));
     XBFS_CUDA(g, cudaMalloc(&g->fb, 3 * ((words + 31) / 32 * 32) * sizeof(unsigned int)));
-    XBFS_CUDA(g, cudaMalloc(&g->qv, 2 * n * sizeof(int)));
-    XBFS_CUDA(g, cudaMalloc(&g->qoff, 2 * n * sizeof(long long)));
-    XBFS_CUDA(g, cudaMalloc(&g->qdelta, 2 * n * sizeof(long long)));
-    XBFS_CUDA(g, cudaMalloc(&g->tile_first, 2 * g->tiles_cap * sizeof(int)));
+    XBFS_CUDA(g, cudaMalloc(&g->qv, 3 * n * sizeof(int)));
+    XBFS_CUDA(g, cudaMalloc(&g->qoff, 3 * n * sizeof(long long)));
+    XBFS_CUDA(g, cudaMalloc(&g->qdelta, 3 * n * sizeof(long long)));
+    XBFS_CUDA(g, cudaMalloc(&g->tile_first, 3 * g->tiles_cap * sizeof(int)));
     XBFS_CUDA(g, cudaMalloc(&g->st, sizeof(DevState)));
     XBFS_CUDA(g, cudaMemset(g->st, 0, sizeof(DevState)));
     XBFS_CUDA(g, cudaMalloc(&g->log, kLogCap * sizeof(LevelRec)));

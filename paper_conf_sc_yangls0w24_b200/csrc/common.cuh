@@ -6,7 +6,7 @@
 //   visited  uint32[W]    W = ceil(N/32); isolated vertices pre-set (never candidates)
 //   fb[3]    uint32[W]    frontier bitmaps, rotated: level k reads fb[k%3] (F_k),
 //                         writes fb[(k+1)%3] (F_{k+1}), clears fb[(k+2)%3] (F_{k-1})
-//   queue[2] {qv int32, qoff int64, qdelta int64}[N] + tile_first int32[A/TILE+2]
+//   queue[3] {qv int32, qoff int64, qdelta int64}[N] + tile_first int32[A/TILE+2]
 //            qoff = exclusive prefix of degrees over the queue (edge-balanced tiles),
 //            qdelta = row_ptr[v] - qoff, so arc a of the frontier is col[a + qdelta[j]].
 //   DevState (device) + HostCtl (pinned, mapped) per handle.
@@ -27,6 +27,12 @@ constexpr int kBuChunkWords = 8;     // bitmap words (256 vertices) per warp chu
 constexpr int kBuBatch = 8;          // arcs probed per lane step (one 32-byte sector of col)
 constexpr int kBuHardMin = 256;      // unresolved rows with more arcs left go warp-cooperative
 constexpr int kGenThreads = 256;
+constexpr int kSmallThreads = 512;   // small-frontier cluster kernel: threads per CTA
+constexpr int kSmallCluster = 8;     // CTAs per cluster (portable size)
+constexpr int kSmallInline = 8;      // frontier vertices with deg <= this are expanded by one thread
+constexpr int kSmallBig = 8192;      // per-CTA list of higher-degree vertices (warp-cooperative)
+constexpr long long kSmallEdgesMax = 9LL * kSmallBig;  // guarantees the big list never overflows
+constexpr int kSmallMaxDeg = 512;    // frontier max degree allowed in the small mode (warp steps <= 16)
 constexpr int kLogCap = 1 << 16;     // per-level log entries kept on the device
 
 struct LevelRec {
@@ -37,6 +43,9 @@ struct LevelRec {
 // Mirror of the scalars the host loop needs after each select (pinned + mapped).
 struct HostCtl {
     int k, strategy, queue_valid, done;
+    long long fsize, fedges;   // |F_k|, edgesF_k of the level about to run
+    unsigned fmaxdeg;          // max degree over F_k
+    int prev_small;            // level k-1 was a small SF level (small-mode entry gate)
 };
 
 struct DevState {
@@ -44,7 +53,10 @@ struct DevState {
     int strategy;           // strategy chosen for level k
     int queue_valid;        // queue buffer k&1 holds F_k
     int done;
-    unsigned long long qctr[2];  // packed (count << dbits) + degree sum, per queue buffer
+    unsigned long long qctr[3];  // packed (count << dbits) + degree sum of the queue of F_k in
+                                 // slot k%3; level k zeroes slot (k+2)%3 (one barrier per level)
+    unsigned qmax[3];            // max degree over the same queue (small-frontier mode gate)
+    unsigned fmaxdeg;            // max degree over F_k
     long long fsize, fedges;     // |F_k|, edgesF_k
     long long fprev;             // |F_{k-1}|
     long long unvisited;         // U_k (non-isolated, unvisited)
@@ -56,6 +68,11 @@ struct DevState {
     double alpha, grow, ratio_min, bu_stay;
     int force, prev_strategy;
     long long source;
+    long long small_edges;       // SF levels with edgesF_k <= this run in the cluster kernel (0 = off)
+    int advanced;                // k_small already advanced the level state: k_select only mirrors it
+    int prev_small;              // level k-1 was a small SF level (small-mode entry gate)
+    int mirror_host;             // host-loop driver: mirror the level state into HostCtl
+    int pad2_;
 };
 
 // Arguments shared by all level kernels (static per handle => graph-capturable).
@@ -67,10 +84,10 @@ struct KArgs {
     const unsigned long long* head;  // per vertex: deg << 32 | first stored neighbour (BU first probe)
     unsigned int* visited;
     unsigned int* fb[3];
-    int* qv[2];
-    long long* qoff[2];
-    long long* qdelta[2];
-    int* tile_first[2];
+    int* qv[3];
+    long long* qoff[3];
+    long long* qdelta[3];
+    int* tile_first[3];
     DevState* st;
     HostCtl* hctl;          // device alias of the mapped host struct
     LevelRec* log;
@@ -100,10 +117,10 @@ struct xbfs_graph {
     // BFS work state
     unsigned int* visited = nullptr;
     unsigned int* fb = nullptr;          // 3 * words
-    int* qv = nullptr;                   // 2 * N
-    long long* qoff = nullptr;           // 2 * N
-    long long* qdelta = nullptr;         // 2 * N
-    int* tile_first = nullptr;           // 2 * tiles_cap
+    int* qv = nullptr;                   // 3 * N (queue of F_k in buffer k%3)
+    long long* qoff = nullptr;           // 3 * N
+    long long* qdelta = nullptr;         // 3 * N
+    int* tile_first = nullptr;           // 3 * tiles_cap
     long long tiles_cap = 0;
     xbfs::DevState* st = nullptr;
     xbfs::LevelRec* log = nullptr;

@@ -18,7 +18,8 @@ from dataclasses import dataclass, field
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libxbfs.so")
+# XBFS_LIB overrides the library path (A/B experiments between builds only).
+LIB_PATH = os.environ.get("XBFS_LIB", os.path.join(_HERE, "libxbfs.so"))
 
 XBFS_OK, XBFS_ERR_INVALID_ARG, XBFS_ERR_OUT_OF_MEMORY, XBFS_ERR_CUDA, XBFS_ERR_NCCL, XBFS_ERR_STATE, \
     XBFS_ERR_UNSUPPORTED = range(7)
@@ -40,7 +41,7 @@ class BuildOpts(ctypes.Structure):
 class RunOpts(ctypes.Structure):
     _fields_ = [("alpha", ctypes.c_double), ("grow", ctypes.c_double), ("ratio_min", ctypes.c_double),
                 ("bu_stay", ctypes.c_double), ("force_strategy", ctypes.c_int32), ("driver", ctypes.c_int32),
-                ("lazy_init", ctypes.c_int32), ("reserved", ctypes.c_int32)]
+                ("small_edges", ctypes.c_int32), ("reserved", ctypes.c_int32)]
 
 
 class RunStats(ctypes.Structure):
@@ -58,7 +59,7 @@ class RunStats(ctypes.Structure):
 
 #: kernel ids of RunStats.kernel_id (XBFS_K_* in include/xbfs.h)
 KERNEL_NAMES = {0: "init_fill", 1: "seed", 2: "generate_pre", 3: "td_expand_sf", 4: "td_expand_ss",
-                5: "generate_post", 6: "bu_traverse", 7: "select"}
+                5: "generate_post", 6: "bu_traverse", 7: "select", 8: "small_sf"}
 
 
 def _load():
@@ -209,10 +210,11 @@ class _StatsBuf:
                       for i in range(min(c.num_kernels, self.kcap))] if self.kcap else [])
 
 
-def make_run_opts(alpha=None, grow=None, ratio_min=None, bu_stay=None, force_strategy=None, driver=None) -> RunOpts:
+def make_run_opts(alpha=None, grow=None, ratio_min=None, bu_stay=None, force_strategy=None, driver=None,
+                  small_edges=None) -> RunOpts:
     o = xbfs_run_opts_default()
     for k, v in dict(alpha=alpha, grow=grow, ratio_min=ratio_min, bu_stay=bu_stay,
-                     force_strategy=force_strategy, driver=driver).items():
+                     force_strategy=force_strategy, driver=driver, small_edges=small_edges).items():
         if v is not None:
             setattr(o, k, v)
     return o

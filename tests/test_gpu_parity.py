@@ -217,3 +217,22 @@ def test_bu_probes_and_parents_match_definition(xb, scale):
                         row = ro.col[ro.row_ptr[v]:ro.row_ptr[v + 1]]
                         assert pa[v] == row[np.argmax(ref[row] == k)]
     g.close()
+
+
+@pytest.mark.parametrize("small", [0, 200, 65536])
+def test_small_frontier_cluster_mode(xb, small):
+    """Small-frontier cluster mode (f3) hands levels back and forth with the
+    level kernels; levels stay bit-exact and stats consistent for any threshold."""
+    for graph in ("grid", "kron"):
+        if graph == "grid":
+            src, dst, n = synth.grid(64, 48, seed=5)
+        else:
+            src, dst, n = synth.kronecker(14, seed=21)
+        og = oracle.build_csr(n, src, dst)
+        g = xb.Graph(_dev(src), _dev(dst), n)
+        roots = [0, n - 1, n // 2] if graph == "grid" else synth.roots(n, src, dst, 5, root_seed=3)
+        for root in roots:
+            for opts in (dict(small_edges=small), dict(small_edges=small, driver=1),
+                         dict(small_edges=small, force_strategy=0), dict(small_edges=small, bu_stay=0.0)):
+                _check_run(g, og, src, dst, root, **opts)
+        g.close()
