@@ -25,11 +25,13 @@ def _declared(header):
 
 
 def test_exports_every_declared_symbol(xb):
-    declared = _declared("xbfs.h")
-    assert declared, "no declarations parsed"
-    for name in declared:
-        assert hasattr(xb.lib, name), f"missing export {name}"
-    assert declared <= set(xb.EXPORTS) | set(getattr(xb, "DIST_EXPORTS", ()))
+    from paper_conf_sc_yangls0w24_b200 import dist
+    for header, listed in (("xbfs.h", xb.EXPORTS), ("xbfs_dist.h", dist.DIST_EXPORTS)):
+        declared = _declared(header)
+        assert declared, f"no declarations parsed from {header}"
+        for name in declared:
+            assert hasattr(xb.lib, name), f"missing export {name}"
+        assert declared == set(listed), (header, declared ^ set(listed))
 
 
 def test_compiled_for_sm100a(xb):
@@ -52,6 +54,11 @@ def test_invalid_arguments_do_not_touch_cuda(xb):
     assert xb.lib.xbfs_reorder(None, 1) == xb.XBFS_ERR_INVALID_ARG
     assert xb.lib.xbfs_graph_info(None, None, None, None, None) == xb.XBFS_ERR_INVALID_ARG
     xb.lib.xbfs_destroy(None)  # NULL-safe
+    from paper_conf_sc_yangls0w24_b200 import dist
+    assert xb.lib.xbfs_dist_build(None, None, 0, 10, 2, 5, None, ctypes.byref(h)) == xb.XBFS_ERR_INVALID_ARG
+    assert xb.lib.xbfs_dist_build(None, None, 0, 10, 0, 0, None, ctypes.byref(h)) == xb.XBFS_ERR_INVALID_ARG
+    assert xb.lib.xbfs_dist_level(None, 0, None) == xb.XBFS_ERR_INVALID_ARG
+    xb.lib.xbfs_dist_destroy(None)
 
 
 def test_product_path_never_imports_oracle():
