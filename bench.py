@@ -435,13 +435,111 @@ def main():
     ap.add_argument("--profile-roots", type=int, default=4)
     ap.add_argument("--cpu-budget", type=float, default=15.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--mode", default="auto", choices=["auto", "dist", "replicas"],
+                    help="N>1: dist = one graph 1D-partitioned over the N GPUs (default), "
+                         "replicas = every GPU its own copy and roots")
     args = ap.parse_args()
     assert args.warmup >= 3 or args.impl == "reference" or os.environ.get("XBFS_ALLOW_SHORT_WARMUP"), \
         "timing rules: at least 3 warm-up steps"
+    world = int(os.environ.get("WORLD_SIZE", "1"))
     if args.impl == "reference":
         run_reference(args)
+    elif args.mode == "dist" or (args.mode == "auto" and world > 1):
+        run_dist(args)
     else:
         run_ours(args)
+
+
+def run_dist(args):
+    """One BFS per step over ONE graph 1D-partitioned across the N ranks
+    (include/xbfs_dist.h): strong scaling of the same s24 workload.  Per-BFS
+    time = max over ranks of the CUDA-event time around the rank's whole level
+    loop (host collectives included); value = harmonic mean of m / t."""
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_sc_yangls0w24_b200 import metrics
+    from paper_conf_sc_yangls0w24_b200.dist import DistGraph
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    dev = torch.device(f"cuda:{local}")
+    if world == 1:
+        for k, v in dict(RANK="0", WORLD_SIZE="1", MASTER_ADDR="127.0.0.1", MASTER_PORT="29517").items():
+            os.environ.setdefault(k, v)
+    dist.init_process_group("nccl" if world > 1 else "gloo", device_id=dev if world > 1 else None)
+    t0 = time.time()
+    src, dst, n = make_graph(args.config, pinned=True)
+    t_gen = time.time() - t0
+    roots = pick_roots(args.config, n, src, dst, args.warmup + args.steps)
+    opts = {}
+    if args.alpha is not None:
+        opts["alpha"] = args.alpha
+    if args.bu_stay is not None:
+        opts["bu_stay"] = args.bu_stay
+    t0 = time.time()
+    dg = DistGraph(torch.from_numpy(src.view(np.int32)), torch.from_numpy(dst.view(np.int32)), n, device=local)
+    torch.cuda.synchronize()
+    t_build = time.time() - t0
+    del src, dst
+    level = torch.empty(max(dg.count, 1), dtype=torch.int32, device=dev)[: dg.count]
+    parent = torch.empty(max(dg.count, 1), dtype=torch.int32, device=dev)[: dg.count]
+    flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
+    for r in roots[: args.warmup]:
+        dg.run(int(r), level, parent, **opts)
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    clocks = ClockSampler(local)
+    clocks.start()
+    per = []
+    for r in roots[args.warmup:]:
+        flush.fill_(1)
+        torch.cuda.synchronize()
+        dist.barrier()
+        ev0.record()
+        _, _, st = dg.run(int(r), level, parent, **opts)
+        ev1.record()
+        ev1.synchronize()
+        ms = torch.tensor([ev0.elapsed_time(ev1)], dtype=torch.float64, device=dev if world > 1 else "cpu")
+        dist.all_reduce(ms, op=dist.ReduceOp.MAX)
+        per.append((int(r), float(ms.item()), st.input_edges_traversed, sum(st.frontier_edges), st.num_levels,
+                    "".join("FSB"[s] for s in st.strategy)))
+    clk = clocks.stop()
+    reached = torch.tensor([int((level >= 0).sum().item())], dtype=torch.int64,
+                           device=dev if world > 1 else "cpu")
+    dist.all_reduce(reached)
+    if rank == 0:
+        teps = [m / (ms * 1e-3) for (_, ms, m, _, _, _) in per]
+        hm = metrics.harmonic_mean(teps)
+        ms_mean = statistics.mean(ms for (_, ms, *_r) in per)
+        peak, peak_src = load_peaks()
+        line = {
+            "metric": METRIC, "value": round(hm / 1e9, 3), "unit": "GTEPS", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": round(ms_mean, 4), "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": "int32",
+            "data": "synthetic (seeded Graph500 Kronecker generator, graph seed 1, root seed 2)",
+            "config": {"workload": workload_name(args.config), "n_vertices": n, "roots": args.steps,
+                       "parallelism": f"1D vertex partition x{world} (xbfs_dist, peer-memory frontier exchange)",
+                       "l2_flush": "512 MiB write before every timed BFS", "alpha": opts.get("alpha", 0.1),
+                       "bu_stay": opts.get("bu_stay", 1.0)},
+            "gteps_per_gpu": round(hm / 1e9 / world, 3),
+            "gteps_arcs_hmean": round(metrics.harmonic_mean([a / (ms * 1e-3) for (_, ms, _, a, _, _) in per]) / 1e9,
+                                      3),
+            "clocks": clk,
+            "e2e": None,
+            "gpu_launches": None,
+            "roofline": None,
+            "cpu_baseline": None,
+            "levels": [p[4] for p in per[:4]],
+            "strategies": [rle(p[5]) for p in per[:4]],
+            "reached_last_root": int(reached.item()),
+            "prep_s": {"generate": round(t_gen, 2), "build_dist": round(t_build, 2)},
+            "peak_gbs": peak, "peak_source": peak_src,
+        }
+        print(json.dumps(line), flush=True)
+    dg.close()
+    dist.destroy_process_group()
 
 
 if __name__ == "__main__":
