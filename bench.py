@@ -169,6 +169,8 @@ def kernel_bytes(name: str, level: int, st, n: int) -> int:
         return metrics.bytes_generate(n, fv, post=False)
     if name == "generate_post":
         return metrics.bytes_generate(n, found, post=True)
+    if name == "ss_count":
+        return metrics.bytes_ss_count(n, found)
     if name == "bu_traverse":
         return metrics.bytes_bu(n, st.unvisited[level], st.bu_probes[level], found)
     return 0

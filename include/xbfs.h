@@ -99,7 +99,8 @@ typedef struct {
 
 /* kernel ids reported in xbfs_run_stats.kernel_id */
 enum { XBFS_K_INIT = 0, XBFS_K_SEED = 1, XBFS_K_GENERATE_PRE = 2, XBFS_K_TD_SF = 3, XBFS_K_TD_SS = 4,
-       XBFS_K_GENERATE_POST = 5, XBFS_K_BU = 6, XBFS_K_SELECT = 7, XBFS_K_SMALL = 8 };
+       XBFS_K_GENERATE_POST = 5, XBFS_K_BU = 6, XBFS_K_SELECT = 7, XBFS_K_SMALL = 8,
+       XBFS_K_SS_COUNT = 9 };
 
 /* Fill opts with the defaults (alpha 0.1, grow 2.0, ratio_min 1e-3, bu_stay 1, adaptive). */
 void xbfs_run_opts_default(xbfs_run_opts* opts);

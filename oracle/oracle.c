@@ -218,11 +218,12 @@ int32_t oracle_select(int64_t f_size, int64_t f_prev, int64_t f_edges, int64_t a
  *   init        : 8n (level+parent) + 5B (visited, non-isolated, 3 frontier maps)
  *   SF step k   : B (stale frontier clear) + 20|F_k| (queue entries) + 4 edgesF_k
  *                 (col) + 44|F_{k+1}| (level 4, parent 4, row_ptr pair 16, queue 20)
- *   SS step k   : B + 20|F_k| + 4 edgesF_k + 8|F_{k+1}|, then the generation scan
- *                 2B + 36|F_{k+1}| (bitmap read, visited OR, row_ptr pair + queue)
+ *   SS step k   : B + 20|F_k| + 4 edgesF_k + 8|F_{k+1}|, then the single scan of
+ *                 the next-frontier bitmap: B + 8|F_{k+1}| (head[] degrees); the
+ *                 queue is rebuilt only if the next step is top-down (below)
  *   BU step k   : 4B (visited read+write, next write, stale clear) + 16|U_k|
  *                 (row_ptr pair per candidate) + 4 probes_k (col) + 8|F_{k+1}|
- *   a TD step right after a BU step first rebuilds the queue: B + 36|F_k|.
+ *   a TD step right after a BU or SS step first rebuilds the queue: B + 36|F_k|.
  * probes(v) = 1 + index of the first level-k neighbour in v's stored row, or
  * deg(v) if none (BU tests only level k: reading C-9).  per_level[k] gets the
  * bytes of step k; the return value includes init. */
@@ -262,9 +263,8 @@ int64_t oracle_byte_replay(int64_t n, const int64_t* row_ptr, const int32_t* col
         } else {
             if (prev_bu) bytes += B + 36 * fsize[k];            /* queue rebuilt from the bitmap */
             bytes += B + 20 * fsize[k] + 4 * fedges[k];
-            if (strategy[k] == 0) bytes += 44 * found;
-            else bytes += 8 * found + 2 * B + 36 * found;       /* single-scan generation */
-            prev_bu = 0;
+            if (strategy[k] == 0) { bytes += 44 * found; prev_bu = 0; }
+            else { bytes += 8 * found + B + 8 * found; prev_bu = 1; }   /* single scan, no queue */
         }
         unvisited -= found;
         if (per_level) per_level[k] = bytes;

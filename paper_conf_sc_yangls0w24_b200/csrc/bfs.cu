@@ -359,6 +359,41 @@ __global__ __launch_bounds__(kExpandThreads, 3) void k_td_expand(KArgs a, int* _
 // bitmap instead of the 4N-byte status array).  role 0: F_k from fb[k%3] into
 // queue k&1 (queue missing after a BU level).  role 1: F_{k+1} from
 // fb[(k+1)%3] into queue (k+1)&1 and visited |= F_{k+1} (after SS expansion).
+// Single-scan's one scan over the status, here the N-bit next-frontier
+// bitmap: it yields the counters the selector needs (|F_{k+1}|, edgesF_{k+1},
+// max degree, from the dense head[] array).  The queue itself is materialised by
+// k_generate(role 0) only if the next level is top-down; a bottom-up next level
+// never needs it (the bitmap is its input).  visited already holds F_{k+1}: the
+// expansion set it with REDs.
+__global__ __launch_bounds__(kGenThreads) void k_ss_count(KArgs a) {
+    count_launch(a.st);
+    const int k = a.st->k;
+    const unsigned int* __restrict__ bm = a.fb[(k + 1) % 3];
+    unsigned long long found = 0, edges = 0;
+    unsigned gmax = 0;
+    for (long long w = blockIdx.x * (long long)blockDim.x + threadIdx.x; w < a.words;
+         w += (long long)gridDim.x * blockDim.x) {
+        const unsigned word = bm[w];
+        if (!word) continue;
+        found += __popc(word);
+        for (unsigned b = word; b; b &= b - 1) {
+            const unsigned d = (unsigned)(__ldg(a.head + w * 32 + __ffs(b) - 1) >> 32);
+            edges += d;
+            gmax = max(gmax, d);
+        }
+    }
+#pragma unroll
+    for (int o = 16; o; o >>= 1) {
+        found += __shfl_xor_sync(FULL, found, o);
+        edges += __shfl_xor_sync(FULL, edges, o);
+    }
+    if ((threadIdx.x & 31) == 0 && found) {
+        atomicAdd(&a.st->acc_found, found);
+        atomicAdd(&a.st->acc_edges, edges);
+    }
+    flush_max(&a.st->qmax[(k + 1) % 3], gmax);
+}
+
 __global__ __launch_bounds__(kGenThreads) void k_generate(KArgs a, int role) {
     count_launch(a.st);
     const int k = a.st->k;
@@ -462,49 +497,76 @@ __global__ __launch_bounds__(kBuThreads, 5) void k_bu_traverse(KArgs a, int* __r
         for (unsigned b = cand; b; b &= b - 1) s_list[wib][pos++] = (int)(w * 32 + __ffs(b) - 1);
         if (lane < kCW) s_found[wib][lane] = 0;
         __syncwarp();
-        // 2. lane-per-candidate, kBuBatch arcs per step in stored (degree-desc) order;
-        //    a lane that finishes takes the next candidate, so lanes stay busy.
-        //    The first probe uses head[v] (deg << 32 | first stored neighbour), a dense
-        //    array read in candidate order; row_ptr/col are touched only on a miss.
+        // 2. first probe of every candidate, kBuFirstIlp candidates per lane in flight:
+        //    head[v] (deg << 32 | first stored neighbour) is a dense array read in
+        //    candidate order, so a hit (the common case after the degree-desc
+        //    re-arrangement) never touches row_ptr or col.  Misses with more
+        //    arcs are compacted in place at the front of s_list.
+        int nmiss = 0;
+        for (int base = 0; base < total; base += 32 * kBuFirstIlp) {
+            int vv[kBuFirstIlp];
+            unsigned long long hv[kBuFirstIlp];
+            unsigned wd[kBuFirstIlp];
+#pragma unroll
+            for (int g = 0; g < kBuFirstIlp; ++g) {
+                const int idx = base + g * 32 + lane;
+                vv[g] = idx < total ? s_list[wib][idx] : -1;
+            }
+#pragma unroll
+            for (int g = 0; g < kBuFirstIlp; ++g) hv[g] = vv[g] >= 0 ? __ldg(a.head + vv[g]) : 0ull;
+#pragma unroll
+            for (int g = 0; g < kBuFirstIlp; ++g) {
+                const int fu = (int)(unsigned)hv[g];
+                wd[g] = vv[g] >= 0 ? __ldcg(cur + (fu >> 5)) : 0u;
+            }
+            __syncwarp();   // every read of this round is done before the in-place compaction
+#pragma unroll
+            for (int g = 0; g < kBuFirstIlp; ++g) {
+                const int v = vv[g];
+                bool miss = false;
+                if (v >= 0) {
+                    const int fu = (int)(unsigned)hv[g];
+                    const long long d = (long long)(hv[g] >> 32);
+                    if ((wd[g] >> (fu & 31)) & 1u) {
+                        level[v] = lvl;
+                        parent[v] = fu;
+                        atomicOr(&s_found[wib][(v >> 5) - c * kCW], 1u << (v & 31));
+                        edges += (unsigned long long)d;
+                        fmax = max(fmax, (unsigned)d);
+                        ++found;
+                        probes += 1;
+                    } else if (d == 1) {
+                        probes += 1;
+                    } else {
+                        miss = true;
+                    }
+                }
+                const unsigned mm = __ballot_sync(FULL, miss);
+                if (miss) s_list[wib][nmiss + __popc(mm & lt)] = v;
+                nmiss += __popc(mm);
+            }
+        }
+        __syncwarp();
+        // 3. the misses: lane-per-candidate, kBuBatch arcs per step in stored
+        //    order from the second arc on; a lane that finishes takes the next
+        //    candidate, so lanes stay busy.
         int v = -1, nxt = 0, nhard = 0;
         long long rs = 0, re = 0, p = 0;
-        unsigned long long hd = 0;
-        bool first = false;
         for (;;) {
             const unsigned need = __ballot_sync(FULL, v < 0);
             if (v < 0) {
                 const int idx = nxt + __popc(need & lt);
-                if (idx < total) {
+                if (idx < nmiss) {
                     v = s_list[wib][idx];
-                    hd = __ldg(a.head + v);
-                    first = true;
+                    rs = a.row_ptr[v];
+                    re = a.row_ptr[v + 1];
+                    p = rs + 1;
                 }
             }
             nxt += __popc(need);
             if (!__any_sync(FULL, v >= 0)) break;
             bool to_hard = false;
-            if (v >= 0 && first) {
-                const int fu = (int)(unsigned)hd;
-                const long long d = (long long)(hd >> 32);
-                if ((__ldcg(cur + (fu >> 5)) >> (fu & 31)) & 1u) {
-                    level[v] = lvl;
-                    parent[v] = fu;
-                    atomicOr(&s_found[wib][(v >> 5) - c * kCW], 1u << (v & 31));
-                    edges += (unsigned long long)d;
-                    fmax = max(fmax, (unsigned)d);
-                    ++found;
-                    probes += 1;
-                    v = -1;
-                } else if (d == 1) {
-                    probes += 1;
-                    v = -1;
-                } else {
-                    rs = a.row_ptr[v];
-                    re = rs + d;
-                    p = rs + 1;
-                    first = false;
-                }
-            } else if (v >= 0) {
+            if (v >= 0) {
                 const long long end = min(re, p + kBuBatch);
                 int u[kBuBatch];
                 unsigned wd[kBuBatch];
@@ -547,7 +609,7 @@ __global__ __launch_bounds__(kBuThreads, 5) void k_bu_traverse(KArgs a, int* __r
             nhard += __popc(hm);
         }
         __syncwarp();
-        // 3. long unresolved rows: the whole warp probes 32 arcs per step, first hit wins
+        // 4. long unresolved rows: the whole warp probes 32 arcs per step, first hit wins
         for (int h = 0; h < nhard; ++h) {
             const int hv = s_hard[wib][h];
             const long long hrs = a.row_ptr[hv], hre = a.row_ptr[hv + 1];
@@ -612,7 +674,7 @@ __global__ void k_select(KArgs a, cudaGraphConditionalHandle h_while) {
     const int k = st->k;
     const int strat = st->strategy;
     long long nf, ne;
-    if (strat == XBFS_BU) {
+    if (strat == XBFS_BU || strat == XBFS_SS) {   // counted by k_bu_traverse / k_ss_count; no queue
         nf = (long long)st->acc_found;
         ne = (long long)st->acc_edges;
         st->queue_valid = 0;
@@ -968,7 +1030,7 @@ xbfs_status launch_level(xbfs_graph* g, const KArgs& a, int* level, int* parent,
     } else if (strat == XBFS_SS) {
         XBFS_LAUNCH(P, XBFS_K_TD_SS, k,
                     (k_td_expand<XBFS_SS><<<G.expand, kExpandThreads, 0, s>>>(a, level, parent)));
-        XBFS_LAUNCH(P, XBFS_K_GENERATE_POST, k, (k_generate<<<G.gen, kGenThreads, 0, s>>>(a, 1)));
+        XBFS_LAUNCH(P, XBFS_K_SS_COUNT, k, (k_ss_count<<<G.gen, kGenThreads, 0, s>>>(a)));
     } else {
         XBFS_LAUNCH(P, XBFS_K_BU, k, (k_bu_traverse<<<G.bu, kBuThreads, 0, s>>>(a, level, parent)));
     }
@@ -1058,13 +1120,14 @@ xbfs_status build_loop_graph(xbfs_graph* g, int* level, int* parent) {
     sp.conditional.size = 6;
     XBFS_CUDA(g, cudaGraphAddNode(&n_sw, body, &n_plan, 1, &sp));
     cudaGraph_t* br = sp.conditional.phGraph_out;
-    int role0 = 0, role1 = 1;
+    int role0 = 0;
     void* a_exp[] = {&a, &level, &parent};
     void* a_gen0[] = {&a, &role0};
-    void* a_gen1[] = {&a, &role1};
     void* f_sf = (void*)k_td_expand<XBFS_SF>;
     void* f_ss = (void*)k_td_expand<XBFS_SS>;
     void* f_gen = (void*)k_generate;
+    void* f_cnt = (void*)k_ss_count;
+    void* a_cnt[] = {&a};
     // 0: SF (queue valid)
     XBFS_TRY(add_kernel(g, br[0], &x, nullptr, f_sf, G.expand, kExpandThreads, a_exp));
     // 1: generate + SF
@@ -1072,11 +1135,11 @@ xbfs_status build_loop_graph(xbfs_graph* g, int* level, int* parent) {
     XBFS_TRY(add_kernel(g, br[1], &y, &x, f_sf, G.expand, kExpandThreads, a_exp));
     // 2: SS + generate (No-Frontier-Generation: the queue exists)
     XBFS_TRY(add_kernel(g, br[2], &x, nullptr, f_ss, G.expand, kExpandThreads, a_exp));
-    XBFS_TRY(add_kernel(g, br[2], &y, &x, f_gen, G.gen, kGenThreads, a_gen1));
+    XBFS_TRY(add_kernel(g, br[2], &y, &x, f_cnt, G.gen, kGenThreads, a_cnt));
     // 3: generate + SS + generate
     XBFS_TRY(add_kernel(g, br[3], &x, nullptr, f_gen, G.gen, kGenThreads, a_gen0));
     XBFS_TRY(add_kernel(g, br[3], &y, &x, f_ss, G.expand, kExpandThreads, a_exp));
-    XBFS_TRY(add_kernel(g, br[3], &x, &y, f_gen, G.gen, kGenThreads, a_gen1));
+    XBFS_TRY(add_kernel(g, br[3], &x, &y, f_cnt, G.gen, kGenThreads, a_cnt));
     // 4: BU
     XBFS_TRY(add_kernel(g, br[4], &x, nullptr, (void*)k_bu_traverse, G.bu, kBuThreads, a_exp));
     // 5: small-frontier cluster mode (cluster dims are compiled into the kernel)

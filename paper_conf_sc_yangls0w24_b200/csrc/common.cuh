@@ -26,6 +26,10 @@ constexpr int kBuThreads = 256;      // bu_traverse block (8 warps)
 constexpr int kBuChunkWords = 8;     // bitmap words (256 vertices) per warp chunk
 constexpr int kBuBatch = 8;          // arcs probed per lane step (one 32-byte sector of col)
 constexpr int kBuHardMin = 256;      // unresolved rows with more arcs left go warp-cooperative
+#ifndef XBFS_BU_FIRST_ILP
+#define XBFS_BU_FIRST_ILP 4
+#endif
+constexpr int kBuFirstIlp = XBFS_BU_FIRST_ILP;  // first probes in flight per lane
 constexpr int kGenThreads = 256;
 constexpr int kSmallThreads = 512;   // small-frontier cluster kernel: threads per CTA
 constexpr int kSmallCluster = 8;     // CTAs per cluster (portable size)

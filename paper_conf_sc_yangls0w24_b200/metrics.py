@@ -84,3 +84,8 @@ def bytes_bu(n: int, unvisited: int, probes: int, found: int) -> int:
     clear) + 16 B row_ptr pair per candidate + 4 B per probed arc + 8 B
     level+parent per found vertex."""
     return 4 * bitmap_bytes(n) + 16 * unvisited + 4 * probes + 8 * found
+
+
+def bytes_ss_count(n: int, found: int) -> int:
+    """Single-scan count pass: next-frontier bitmap read + 8 B head[] per vertex."""
+    return bitmap_bytes(n) + 8 * found

@@ -59,7 +59,8 @@ class RunStats(ctypes.Structure):
 
 #: kernel ids of RunStats.kernel_id (XBFS_K_* in include/xbfs.h)
 KERNEL_NAMES = {0: "init_fill", 1: "seed", 2: "generate_pre", 3: "td_expand_sf", 4: "td_expand_ss",
-                5: "generate_post", 6: "bu_traverse", 7: "select", 8: "small_sf"}
+                5: "generate_post", 6: "bu_traverse", 7: "select", 8: "small_sf",
+                9: "ss_count"}
 
 
 def _load():

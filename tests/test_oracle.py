@@ -321,7 +321,8 @@ def test_byte_replay_hand_computed():
       L2 SF     rebuild queue after BU: B + 36*|F2| = 40; then
                 B + 20 + 4*edgesF2(2) + 44*|F3|                   = 40+4+20+8+44 = 116
       L3 SF     B + 20 + 4*1 + 0                                  = 28
-    SS variant at L2: 40 + (4 + 20 + 8 + 8*1) + (8 + 36*1)       = 124
+    SS variant at L2: 40 + (4 + 20 + 8 + 8*1) + (4 + 8*1)         = 92
+    and the SF step after it rebuilds the queue again: 40 + 28    = 68
     """
     n, src, dst = _graph(4, [(0, 1), (1, 2), (2, 3)])
     g = oracle.reorder(oracle.build_csr(n, src, dst))
@@ -331,7 +332,7 @@ def test_byte_replay_hand_computed():
     assert per.tolist() == [72, 64, 116, 28]
     assert tot == 52 + 72 + 64 + 116 + 28
     _, per2 = oracle.byte_replay(g, level, [0, 2, 1, 0])
-    assert per2[2] == 124
+    assert per2[2] == 92 and per2[3] == 68
 
 
 # ------------------------------------------------------- paper byte model pin
