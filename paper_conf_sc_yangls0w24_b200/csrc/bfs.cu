@@ -190,11 +190,12 @@ __global__ __launch_bounds__(256) void k_init_fill(KArgs a, int* __restrict__ le
 __device__ int choose_strategy(const DevState* st, long long arcs, long long fsize, long long fprev,
                                long long fedges, long long unvisited, int prev) {
     if (st->force >= 0) return st->force;
-    const double ratio = arcs > 0 ? (double)fedges / (double)arcs : 0.0;
-    if (ratio > st->alpha) return XBFS_BU;                                    // P:L87, strict (C-8)
-    if (st->bu_stay > 0.0 && prev == XBFS_BU && (double)unvisited * st->bu_stay < (double)fedges)
+    // ratio = edgesF / A compared as edgesF > alpha * A (no division on the critical path)
+    const double e = (double)fedges, A = (double)arcs;
+    if (arcs > 0 && e > st->alpha * A) return XBFS_BU;                        // P:L87, strict (C-8)
+    if (st->bu_stay > 0.0 && prev == XBFS_BU && (double)unvisited * st->bu_stay < e)
         return XBFS_BU;                                                       // C-11 (optional)
-    if ((double)fsize > st->grow * (double)fprev && ratio > st->ratio_min) return XBFS_SS;  // C-10
+    if ((double)fsize > st->grow * (double)fprev && arcs > 0 && e > st->ratio_min * A) return XBFS_SS;  // C-10
     return XBFS_SF;
 }
 
@@ -237,6 +238,64 @@ __global__ void k_seed(KArgs a, int* level, int* parent, long long nonisolated_c
     st->source = s;
     st->prev_strategy = -1;
     st->strategy = choose_strategy(st, a.arcs, 1, 0, deg, st->unvisited, -1);
+    mirror_host(a, st);
+}
+
+// ------------------------------------------------------------- select
+// End of level k: consolidate the counters, log the level, choose the strategy of
+// level k+1 (P:L87 rule + readings C-10/C-11) and rotate the counter slots.
+// One thread (k_select).  Fusing it into the last block of the level kernels was
+// measured slower: it raised their register pressure (spills).
+__device__ void select_body(const KArgs& a) {
+    // one parallel read of the whole state (independent loads in flight together),
+    // then plain stores: the selector is on the critical path of every level
+    DevState local = *a.st;
+    DevState* st = &local;
+    const int k = st->k;
+    const int strat = st->strategy;
+    long long nf, ne;
+    if (strat == XBFS_BU || strat == XBFS_SS) {   // counted by k_bu_traverse / k_ss_count; no queue
+        nf = (long long)st->acc_found;
+        ne = (long long)st->acc_edges;
+        st->queue_valid = 0;
+    } else {
+        const unsigned long long q = st->qctr[(k + 1) % 3];
+        nf = (long long)(q >> a.dbits);
+        ne = (long long)(q & ((1ull << a.dbits) - 1ull));
+        st->queue_valid = 1;
+    }
+    if (k < kLogCap) {
+        LevelRec r;
+        r.fsize = st->fsize;
+        r.fedges = st->fedges;
+        r.unvisited = st->unvisited;
+        r.probes = strat == XBFS_BU ? (long long)st->acc_probes : 0;
+        r.strategy = strat;
+        r.pad = 0;
+        a.log[k] = r;
+    }
+    // enter the small-frontier mode only after one small SF level has already run
+    // through the level kernels (a single small level does not pay for the switch)
+    st->prev_small = strat == XBFS_SF && st->fedges <= st->small_edges && st->fmaxdeg <= (unsigned)kSmallMaxDeg;
+    st->reached += st->fsize;
+    st->arcs_traversed += st->fedges;
+    st->fprev = st->fsize;
+    st->fsize = nf;
+    st->fedges = ne;
+    st->unvisited -= nf;
+    st->acc_found = st->acc_edges = st->acc_probes = 0;
+    st->prev_strategy = strat;
+    st->k = k + 1;
+    st->fmaxdeg = st->qmax[(k + 1) % 3];
+    st->qctr[(k + 2) % 3] = 0;   // counter of the queue built during level k+1
+    st->qmax[(k + 2) % 3] = 0;
+    if (nf == 0) {
+        st->done = 1;
+        st->nlevels = k + 1;
+    } else {
+        st->strategy = choose_strategy(st, a.arcs, nf, st->fprev, ne, st->unvisited, strat);
+    }
+    *a.st = local;
     mirror_host(a, st);
 }
 
@@ -671,51 +730,7 @@ __global__ void k_select(KArgs a, cudaGraphConditionalHandle h_while) {
         if (kGraph) cudaGraphSetConditional(h_while, st->done ? 0u : 1u);
         return;
     }
-    const int k = st->k;
-    const int strat = st->strategy;
-    long long nf, ne;
-    if (strat == XBFS_BU || strat == XBFS_SS) {   // counted by k_bu_traverse / k_ss_count; no queue
-        nf = (long long)st->acc_found;
-        ne = (long long)st->acc_edges;
-        st->queue_valid = 0;
-    } else {
-        const unsigned long long q = st->qctr[(k + 1) % 3];
-        nf = (long long)(q >> a.dbits);
-        ne = (long long)(q & ((1ull << a.dbits) - 1ull));
-        st->queue_valid = 1;
-    }
-    if (k < kLogCap) {
-        LevelRec r;
-        r.fsize = st->fsize;
-        r.fedges = st->fedges;
-        r.unvisited = st->unvisited;
-        r.probes = strat == XBFS_BU ? (long long)st->acc_probes : 0;
-        r.strategy = strat;
-        r.pad = 0;
-        a.log[k] = r;
-    }
-    // enter the small-frontier mode only after one small SF level has already run
-    // through the level kernels (a single small level does not pay for the switch)
-    st->prev_small = strat == XBFS_SF && st->fedges <= st->small_edges && st->fmaxdeg <= (unsigned)kSmallMaxDeg;
-    st->reached += st->fsize;
-    st->arcs_traversed += st->fedges;
-    st->fprev = st->fsize;
-    st->fsize = nf;
-    st->fedges = ne;
-    st->unvisited -= nf;
-    st->acc_found = st->acc_edges = st->acc_probes = 0;
-    st->prev_strategy = strat;
-    st->k = k + 1;
-    st->fmaxdeg = st->qmax[(k + 1) % 3];
-    st->qctr[(k + 2) % 3] = 0;   // counter of the queue built during level k+1
-    st->qmax[(k + 2) % 3] = 0;
-    if (nf == 0) {
-        st->done = 1;
-        st->nlevels = k + 1;
-    } else {
-        st->strategy = choose_strategy(st, a.arcs, nf, st->fprev, ne, st->unvisited, strat);
-    }
-    mirror_host(a, st);
+    select_body(a);
     if (kGraph) cudaGraphSetConditional(h_while, st->done ? 0u : 1u);
 }
 
@@ -904,7 +919,7 @@ __global__ void __cluster_dims__(kSmallCluster, 1, 1) __launch_bounds__(kSmallTh
         st->prev_strategy = XBFS_SF;
         st->acc_found = st->acc_edges = st->acc_probes = 0;
         st->fmaxdeg = fmaxdeg;
-        st->advanced = 1;
+        st->advanced = st->mirror_host ? 0 : 1;   // graph driver: its k_select node only mirrors
         st->prev_small = 1;
         mirror_host(a, st);
     }
@@ -1017,9 +1032,9 @@ xbfs_status launch_level(xbfs_graph* g, const KArgs& a, int* level, int* parent,
                          Prof& P) {
     const Grids G = grids_for(g);
     cudaStream_t s = g->stream;
+    // The small-frontier kernel advances the level state itself (no k_select).
     if (prev_small && small_gate(small_edges, strat, queue_valid, fedges, maxdeg)) {
         XBFS_LAUNCH(P, XBFS_K_SMALL, k, (k_small_sf<<<kSmallCluster, kSmallThreads, 0, s>>>(a, level, parent)));
-        XBFS_LAUNCH(P, XBFS_K_SELECT, k, (k_select<false><<<1, 1, 0, s>>>(a, 0)));
         return XBFS_OK;
     }
     if (strat != XBFS_BU && !queue_valid)
@@ -1122,6 +1137,7 @@ xbfs_status build_loop_graph(xbfs_graph* g, int* level, int* parent) {
     cudaGraph_t* br = sp.conditional.phGraph_out;
     int role0 = 0;
     void* a_exp[] = {&a, &level, &parent};
+    void* a_small[] = {&a, &level, &parent};
     void* a_gen0[] = {&a, &role0};
     void* f_sf = (void*)k_td_expand<XBFS_SF>;
     void* f_ss = (void*)k_td_expand<XBFS_SS>;
@@ -1143,7 +1159,7 @@ xbfs_status build_loop_graph(xbfs_graph* g, int* level, int* parent) {
     // 4: BU
     XBFS_TRY(add_kernel(g, br[4], &x, nullptr, (void*)k_bu_traverse, G.bu, kBuThreads, a_exp));
     // 5: small-frontier cluster mode (cluster dims are compiled into the kernel)
-    XBFS_TRY(add_kernel(g, br[5], &x, nullptr, (void*)k_small_sf, kSmallCluster, kSmallThreads, a_exp));
+    XBFS_TRY(add_kernel(g, br[5], &x, nullptr, (void*)k_small_sf, kSmallCluster, kSmallThreads, a_small));
     {
         void* args[] = {&a, &h_while};
         XBFS_TRY(add_kernel(g, body, &n_sel, &n_sw, (void*)k_select<true>, 1, 1, args));
