@@ -68,7 +68,9 @@ typedef struct {
     int32_t driver;          /* 0 auto, 1 host loop (one sync per level), 2 CUDA-graph device loop */
     int32_t small_edges;     /* SF levels with edgesF_k <= this run inside one thread-block cluster
                                 (small-frontier mode); default 65536, 0 = off, max 73728 */
-    int32_t reserved;
+    int32_t plan_len;        /* > 0: strategy plan for levels [0, plan_len) (host-loop driver only) */
+    const int8_t* plan;      /* host array: plan[k] in {-1 selector, 0 SF, 1 SS, 2 BU} overrides the
+                                strategy of level k (forced-strategy studies, Tab VI) */
 } xbfs_run_opts;
 
 /* Per-run statistics; filled when a non-NULL pointer is passed (xbfs_run then

@@ -1054,15 +1054,24 @@ xbfs_status launch_level(xbfs_graph* g, const KArgs& a, int* level, int* parent,
 }
 
 xbfs_status run_host_loop(xbfs_graph* g, const KArgs& a, int* level, int* parent, long long small_edges,
-                          Prof& P) {
+                          const int8_t* plan, int plan_len, Prof& P) {
     // k_seed wrote hctl; wait for it, then one sync per level (P:L151's
     // host/device crossing, kept as the debug / measurement driver).
     XBFS_CUDA(g, cudaStreamSynchronize(g->stream));
     for (;;) {
         volatile HostCtl* h = g->hctl;
         if (h->done) break;
-        XBFS_TRY(launch_level(g, a, level, parent, h->k, h->strategy, h->queue_valid, h->fedges, h->fmaxdeg,
-                              h->prev_small,
+        int strat = h->strategy, prev_small = h->prev_small;
+        const int k = h->k;
+        if (k < plan_len) {
+            prev_small = 0;   // planned levels always run through the level kernels
+            if (plan[k] >= 0 && plan[k] != strat) {
+                strat = plan[k];
+                XBFS_CUDA(g, cudaMemcpyAsync(&g->st->strategy, &strat, sizeof(int), cudaMemcpyHostToDevice,
+                                             g->stream));
+            }
+        }
+        XBFS_TRY(launch_level(g, a, level, parent, k, strat, h->queue_valid, h->fedges, h->fmaxdeg, prev_small,
                               small_edges, P));
         XBFS_CUDA(g, cudaStreamSynchronize(g->stream));
     }
@@ -1192,7 +1201,8 @@ static xbfs_status run_impl(xbfs_graph* g, int64_t source, int32_t* level, int32
     XBFS_CUDA(g, cudaSetDevice(g->device));
 
     KArgs a = g->kargs();
-    const bool use_graph = (o.driver == 0 || o.driver == 2) && !(stats && stats->kernel_capacity > 0);
+    const bool use_graph = (o.driver == 0 || o.driver == 2) && !(stats && stats->kernel_capacity > 0) &&
+                           !(o.plan && o.plan_len > 0);
     // selection parameters live in the device state
     {
         DevState hs;
@@ -1222,7 +1232,8 @@ static xbfs_status run_impl(xbfs_graph* g, int64_t source, int32_t* level, int32
                 (k_init_fill<<<G.init, 256, 0, g->stream>>>(a, level, parent, g->nonisolated)));
     XBFS_LAUNCH(P, XBFS_K_SEED, -1,
                 (k_seed<<<1, 1, 0, g->stream>>>(a, level, parent, g->nonisolated_count)));
-    XBFS_TRY(run_host_loop(g, a, level, parent, std::min<long long>(std::max(o.small_edges, 0), kSmallEdgesMax), P));
+    XBFS_TRY(run_host_loop(g, a, level, parent, std::min<long long>(std::max(o.small_edges, 0), kSmallEdgesMax),
+                           o.plan, o.plan ? std::max(o.plan_len, 0) : 0, P));
     XBFS_CUDA(g, cudaEventRecord(g->ev1, g->stream));
     }
 

@@ -41,7 +41,8 @@ class BuildOpts(ctypes.Structure):
 class RunOpts(ctypes.Structure):
     _fields_ = [("alpha", ctypes.c_double), ("grow", ctypes.c_double), ("ratio_min", ctypes.c_double),
                 ("bu_stay", ctypes.c_double), ("force_strategy", ctypes.c_int32), ("driver", ctypes.c_int32),
-                ("small_edges", ctypes.c_int32), ("reserved", ctypes.c_int32)]
+                ("small_edges", ctypes.c_int32), ("plan_len", ctypes.c_int32),
+                ("plan", ctypes.POINTER(ctypes.c_int8))]
 
 
 class RunStats(ctypes.Structure):
@@ -212,12 +213,18 @@ class _StatsBuf:
 
 
 def make_run_opts(alpha=None, grow=None, ratio_min=None, bu_stay=None, force_strategy=None, driver=None,
-                  small_edges=None) -> RunOpts:
+                  small_edges=None, plan=None) -> RunOpts:
+    """plan: sequence of per-level strategies (-1 = selector, 0 SF, 1 SS, 2 BU)."""
     o = xbfs_run_opts_default()
     for k, v in dict(alpha=alpha, grow=grow, ratio_min=ratio_min, bu_stay=bu_stay,
                      force_strategy=force_strategy, driver=driver, small_edges=small_edges).items():
         if v is not None:
             setattr(o, k, v)
+    if plan is not None and len(plan):
+        arr = (ctypes.c_int8 * len(plan))(*[int(x) for x in plan])
+        o._plan_keepalive = arr
+        o.plan = ctypes.cast(arr, ctypes.POINTER(ctypes.c_int8))
+        o.plan_len = len(plan)
     return o
 
 

@@ -236,3 +236,20 @@ def test_small_frontier_cluster_mode(xb, small):
                          dict(small_edges=small, force_strategy=0), dict(small_edges=small, bu_stay=0.0)):
                 _check_run(g, og, src, dst, root, **opts)
         g.close()
+
+
+def test_per_level_strategy_plan(xb):
+    """A per-level plan (forced-strategy studies) is followed level by level,
+    including random mixes of SF/SS/BU; levels stay exact."""
+    src, dst, n = synth.kronecker(14, seed=8)
+    og = oracle.build_csr(n, src, dst)
+    g = xb.Graph(_dev(src), _dev(dst), n)
+    rng = np.random.default_rng(1)
+    for root in synth.roots(n, src, dst, 4, root_seed=13):
+        for _ in range(4):
+            plan = rng.integers(0, 3, 12).tolist()
+            st = _check_run(g, og, src, dst, root, plan=plan)
+            assert st.strategy == plan[:st.num_levels]
+        st = _check_run(g, og, src, dst, root, plan=[-1, 2, -1])
+        assert st.strategy[1] == 2
+    g.close()
