@@ -1,0 +1,202 @@
+// bu_core.cuh — the bottom-up step over a range of owned bitmap words, shared
+// by the single-GPU kernel (k_bu_traverse, bfs.cu) and the multi-GPU one
+// (dist.cu).  P:L122-131 §III-C; design notes in bfs.cu / DESIGN.md §5.
+#pragma once
+#include "common.cuh"
+
+namespace xbfs {
+
+// What a BU step reads and writes.  Vertex indices are LOCAL (the owned range
+// starts at 0); col values and the frontier bitmap `cur` are GLOBAL.
+struct BuView {
+    const unsigned int* cur;          // F_k, global bitmap
+    unsigned int* visited;            // owned words
+    long long words;                  // owned words
+    const unsigned long long* head;   // owned: deg << 32 | first stored neighbour
+    const long long* row_ptr;         // owned rows
+    const int* col;
+    int* level;                       // owned
+    int* parent;                      // owned (global ids)
+    int lvl;                          // k + 1
+};
+
+// publish(w, vis, found_word): store the owned word w of F_{k+1} and update visited.
+template <class Publish>
+__device__ __forceinline__ void bu_chunks(const BuView& b, Publish publish, unsigned long long& found,
+                                          unsigned long long& edges, unsigned long long& probes, unsigned& fmax) {
+    constexpr unsigned FULL = 0xffffffffu;
+    const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+    const unsigned lt = (1u << lane) - 1u;
+    constexpr int kCW = kBuChunkWords, kCV = kBuChunkWords * 32;
+    __shared__ int s_list[kBuThreads / 32][kCV];   // candidates of the warp's chunk
+    __shared__ int s_hard[kBuThreads / 32][kCV];   // long unresolved rows (warp-cooperative)
+    __shared__ int s_hoff[kBuThreads / 32][kCV];   // arcs already probed for each hard row
+    __shared__ unsigned s_found[kBuThreads / 32][kCW];
+    const long long nchunks = (b.words + kCW - 1) / kCW;
+    const long long gw = (blockIdx.x * (long long)blockDim.x + threadIdx.x) >> 5;
+    const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
+    for (long long c = gw; c < nchunks; c += nw) {
+        // 1. candidates of kCW bitmap words: ballot/popc compaction into shared memory
+        //    (the paper's count + prefix-sum + queue-write "double scan").
+        const long long w = c * kCW + lane;
+        const bool own = lane < kCW && w < b.words;
+        const unsigned vis = own ? b.visited[w] : FULL;
+        const unsigned cand = ~vis;
+        const int cnt = __popc(cand);
+        int incl = cnt;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const int t = __shfl_up_sync(FULL, incl, o);
+            if (lane >= o) incl += t;
+        }
+        const int total = __shfl_sync(FULL, incl, 31);
+        int pos = incl - cnt;
+        for (unsigned bits = cand; bits; bits &= bits - 1) s_list[wib][pos++] = (int)(w * 32 + __ffs(bits) - 1);
+        if (lane < kCW) s_found[wib][lane] = 0;
+        __syncwarp();
+        // 2. first probe of every candidate, kBuFirstIlp candidates per lane in flight:
+        //    head[v] (deg << 32 | first stored neighbour) is a dense array read in
+        //    candidate order, so a hit (the common case after the degree-desc
+        //    re-arrangement) never touches row_ptr or col.  Misses with more
+        //    arcs are compacted in place at the front of s_list.
+        int nmiss = 0;
+        for (int base = 0; base < total; base += 32 * kBuFirstIlp) {
+            int vv[kBuFirstIlp];
+            unsigned long long hv[kBuFirstIlp];
+            unsigned wd[kBuFirstIlp];
+#pragma unroll
+            for (int g = 0; g < kBuFirstIlp; ++g) {
+                const int idx = base + g * 32 + lane;
+                vv[g] = idx < total ? s_list[wib][idx] : -1;
+            }
+#pragma unroll
+            for (int g = 0; g < kBuFirstIlp; ++g) hv[g] = vv[g] >= 0 ? __ldg(b.head + vv[g]) : 0ull;
+#pragma unroll
+            for (int g = 0; g < kBuFirstIlp; ++g) {
+                const int fu = (int)(unsigned)hv[g];
+                wd[g] = vv[g] >= 0 ? __ldcg(b.cur + (fu >> 5)) : 0u;
+            }
+            __syncwarp();   // every read of this round is done before the in-place compaction
+#pragma unroll
+            for (int g = 0; g < kBuFirstIlp; ++g) {
+                const int v = vv[g];
+                bool miss = false;
+                if (v >= 0) {
+                    const int fu = (int)(unsigned)hv[g];
+                    const long long d = (long long)(hv[g] >> 32);
+                    if ((wd[g] >> (fu & 31)) & 1u) {
+                        b.level[v] = b.lvl;
+                        b.parent[v] = fu;
+                        atomicOr(&s_found[wib][(v >> 5) - c * kCW], 1u << (v & 31));
+                        edges += (unsigned long long)d;
+                        fmax = max(fmax, (unsigned)d);
+                        ++found;
+                        probes += 1;
+                    } else if (d == 1) {
+                        probes += 1;
+                    } else {
+                        miss = true;
+                    }
+                }
+                const unsigned mm = __ballot_sync(FULL, miss);
+                if (miss) s_list[wib][nmiss + __popc(mm & lt)] = v;
+                nmiss += __popc(mm);
+            }
+        }
+        __syncwarp();
+        // 3. the misses: lane-per-candidate, kBuBatch arcs per step in stored
+        //    order from the second arc on; a lane that finishes takes the next
+        //    candidate, so lanes stay busy.
+        int v = -1, nxt = 0, nhard = 0;
+        long long rs = 0, re = 0, p = 0;
+        for (;;) {
+            const unsigned need = __ballot_sync(FULL, v < 0);
+            if (v < 0) {
+                const int idx = nxt + __popc(need & lt);
+                if (idx < nmiss) {
+                    v = s_list[wib][idx];
+                    rs = b.row_ptr[v];
+                    re = b.row_ptr[v + 1];
+                    p = rs + 1;
+                }
+            }
+            nxt += __popc(need);
+            if (!__any_sync(FULL, v >= 0)) break;
+            bool to_hard = false;
+            if (v >= 0) {
+                const long long end = min(re, p + kBuBatch);
+                int u[kBuBatch];
+                unsigned wd[kBuBatch];
+#pragma unroll
+                for (int j = 0; j < kBuBatch; ++j) u[j] = (p + j < end) ? __ldg(b.col + p + j) : -1;
+#pragma unroll
+                for (int j = 0; j < kBuBatch; ++j) wd[j] = u[j] >= 0 ? __ldcg(b.cur + (u[j] >> 5)) : 0u;
+                int hit = -1;
+#pragma unroll
+                for (int j = kBuBatch - 1; j >= 0; --j)
+                    if (u[j] >= 0 && ((wd[j] >> (u[j] & 31)) & 1u)) hit = j;   // first hit in row order
+                if (hit >= 0) {
+                    int pu = u[0];
+#pragma unroll
+                    for (int j = 1; j < kBuBatch; ++j) if (j == hit) pu = u[j];
+                    b.level[v] = b.lvl;
+                    b.parent[v] = pu;
+                    atomicOr(&s_found[wib][(v >> 5) - c * kCW], 1u << (v & 31));
+                    edges += (unsigned long long)(re - rs);
+                    fmax = max(fmax, (unsigned)(re - rs));
+                    ++found;
+                    probes += (unsigned long long)(p + hit + 1 - rs);
+                    v = -1;
+                } else if (end == re) {
+                    probes += (unsigned long long)(re - rs);
+                    v = -1;
+                } else if (re - end > kBuHardMin) {
+                    to_hard = true;
+                } else {
+                    p = end;
+                }
+            }
+            const unsigned hm = __ballot_sync(FULL, to_hard);
+            if (to_hard) {
+                const int hi = nhard + __popc(hm & lt);
+                s_hard[wib][hi] = v;
+                s_hoff[wib][hi] = (int)(p + kBuBatch - rs);
+                v = -1;
+            }
+            nhard += __popc(hm);
+        }
+        __syncwarp();
+        // 4. long unresolved rows: the whole warp probes 32 arcs per step, first hit wins
+        for (int h = 0; h < nhard; ++h) {
+            const int hv = s_hard[wib][h];
+            const long long hrs = b.row_ptr[hv], hre = b.row_ptr[hv + 1];
+            bool hit_any = false;
+            for (long long base = hrs + s_hoff[wib][h]; base < hre; base += 32) {
+                const long long pp = base + lane;
+                const int u = pp < hre ? __ldg(b.col + pp) : -1;
+                const bool hit = u >= 0 && ((__ldcg(b.cur + (u >> 5)) >> (u & 31)) & 1u);
+                const unsigned m = __ballot_sync(FULL, hit);
+                if (m) {
+                    const int first = __ffs(m) - 1;
+                    if (lane == first) {
+                        b.level[hv] = b.lvl;
+                        b.parent[hv] = u;
+                        atomicOr(&s_found[wib][(hv >> 5) - c * kCW], 1u << (hv & 31));
+                        edges += (unsigned long long)(hre - hrs);
+                        fmax = max(fmax, (unsigned)(hre - hrs));
+                        ++found;
+                        probes += (unsigned long long)(pp + 1 - hrs);
+                    }
+                    hit_any = true;
+                    break;
+                }
+            }
+            if (!hit_any && lane == 0) probes += (unsigned long long)(hre - hrs);
+        }
+        __syncwarp();
+        if (own) publish(w, vis, s_found[wib][lane]);
+        __syncwarp();
+    }
+}
+
+}  // namespace xbfs

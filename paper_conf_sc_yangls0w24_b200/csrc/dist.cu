@@ -13,6 +13,7 @@
 #include <new>
 #include <vector>
 
+#include "bu_core.cuh"
 #include "common.cuh"
 #include "xbfs_dist.h"
 
@@ -110,37 +111,33 @@ __device__ __forceinline__ int find_parent(const DArgs& a, const unsigned* cur, 
 }
 
 // ---------------------------------------------------------------- BU
-// Lane per owned bitmap word: its unvisited vertices probe F_k (local replica).
-__global__ __launch_bounds__(kB) void k_bu(DArgs a, int k) {
-    const unsigned* cur = a.fb[k % 3];
+// The single-GPU bottom-up core (bu_core.cuh) over the owned words; each owned
+// word of F_{k+1} is published to every replica by the lane that owns it.
+__global__ __launch_bounds__(kBuThreads, 5) void k_bu(DArgs a, int k) {
     const int slot = (k + 1) % 3;
-    const int lvl = k + 1;
     unsigned long long found = 0, edges = 0, m = 0, probes = 0;
+    unsigned fmax = 0;
     // stale replica clear (F_{k-1}), full N bits, local only
     for (long long w = blockIdx.x * (long long)blockDim.x + threadIdx.x; w < a.fwords;
          w += (long long)gridDim.x * blockDim.x)
         a.fb[(k + 2) % 3][w] = 0;
-    for (long long w = blockIdx.x * (long long)blockDim.x + threadIdx.x; w < a.cw;
-         w += (long long)gridDim.x * blockDim.x) {
-        const unsigned vis = a.vis[w];
-        unsigned f = 0;
-        for (unsigned b = ~vis; b; b &= b - 1) {
-            const int bit = __ffs(b) - 1;
-            const long long vl = w * 32 + bit;
-            const int par = find_parent(a, cur, vl, probes);
-            if (par >= 0) {
-                a.level[vl] = lvl;
-                a.parent[vl] = par;
-                f |= 1u << bit;
-                const unsigned long long hd = __ldg(a.head + vl);
-                edges += hd >> 32;
-                m += (unsigned long long)a.tcount[vl];
-                ++found;
-            }
-        }
-        if (f) a.vis[w] = vis | f;
+    BuView b;
+    b.cur = a.fb[k % 3];
+    b.visited = a.vis;
+    b.words = a.cw;
+    b.head = a.head;
+    b.row_ptr = a.row_ptr;
+    b.col = a.col;
+    b.level = a.level;
+    b.parent = a.parent;
+    b.lvl = k + 1;
+    bu_chunks(b, [&](long long w, unsigned vis, unsigned f) {
         publish_word(a, slot, w, f);
-    }
+        if (f) {
+            a.vis[w] = vis | f;
+            for (unsigned bits = f; bits; bits &= bits - 1) m += (unsigned long long)a.tcount[w * 32 + __ffs(bits) - 1];
+        }
+    }, found, edges, probes, fmax);
     for (int o = 16; o; o >>= 1) {
         found += __shfl_xor_sync(FULL, found, o);
         edges += __shfl_xor_sync(FULL, edges, o);
@@ -763,7 +760,9 @@ xbfs_status xbfs_dist_level(xbfs_dist* d, int32_t phase, int64_t counts[XBFS_DIS
     if (d->strategy == XBFS_BU) {
         if (phase == 0) {
             DCUDA(d, cudaMemsetAsync(d->acc, 0, sizeof(DAcc), d->stream));
-            k_bu<<<grid, kB, 0, d->stream>>>(a, k);
+            int nsm = 148;
+            cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, d->device);
+            k_bu<<<nsm * 5, kBuThreads, 0, d->stream>>>(a, k);
             DCUDA(d, cudaGetLastError());
         }
     } else if (phase == 0) {
