@@ -42,6 +42,9 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, Publish publish, unsi
         const bool own = lane < kCW && w < b.words;
         const unsigned vis = own ? b.visited[w] : FULL;
         const unsigned cand = ~vis;
+        // fast path: no candidate in the chunk (most chunks in late BU levels); F_{k+1}
+        // words start out zero (the stale-bitmap clear of level k-1), so nothing to write
+        if (__ballot_sync(FULL, cand != 0u) == 0u) continue;
         const int cnt = __popc(cand);
         int incl = cnt;
 #pragma unroll
@@ -194,7 +197,10 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, Publish publish, unsi
             if (!hit_any && lane == 0) probes += (unsigned long long)(hre - hrs);
         }
         __syncwarp();
-        if (own) publish(w, vis, s_found[wib][lane]);
+        if (own) {
+            const unsigned f = s_found[wib][lane];
+            if (f) publish(w, vis, f);   // zero words are already zero in every replica
+        }
         __syncwarp();
     }
 }

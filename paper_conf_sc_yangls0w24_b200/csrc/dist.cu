@@ -253,7 +253,7 @@ __global__ __launch_bounds__(kB) void k_merge(DArgs a, int k) {
             m += (unsigned long long)a.tcount[vl];
             ++found;
         }
-        publish_word(a, slot, w, fin);
+        if (fin) publish_word(a, slot, w, fin);   // zero words are zero in every replica
     }
     for (int o = 16; o; o >>= 1) {
         found += __shfl_xor_sync(FULL, found, o);
