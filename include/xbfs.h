@@ -65,7 +65,10 @@ typedef struct {
     double ratio_min;        /*   "                                                    */
     double bu_stay;          /* >0: stay BU while |U_k| * bu_stay < edgesF_k (C-11); default 1.0, 0 = paper rule */
     int32_t force_strategy;  /* -1 adaptive; 0 SF, 1 SS, 2 BU on every level (tests, Fig 7 sweep) */
-    int32_t driver;          /* 0 auto, 1 host loop (one sync per level), 2 CUDA-graph device loop */
+    int32_t driver;          /* 0 auto (= 3), 1 host loop (one sync per level), 2 CUDA-graph device
+                                loop, 3 persistent kernel (one cooperative launch per BFS, grid
+                                barriers between levels).  Per-launch profiling and plans always
+                                use the host loop. */
     int32_t small_edges;     /* SF levels with edgesF_k <= this run inside one thread-block cluster
                                 (small-frontier mode); default 65536, 0 = off, max 73728 */
     int32_t plan_len;        /* > 0: strategy plan for levels [0, plan_len) (host-loop driver only) */
@@ -97,6 +100,9 @@ typedef struct {
     int32_t* kernel_id;            /* XBFS_K_* */
     int32_t* kernel_level;         /* level k the launch belongs to (-1 = init) */
     float* kernel_ms;              /* event-timed duration */
+    /* [level_capacity] device time of level k in ms (persistent driver: %globaltimer
+     * stamps at the grid barrier ending each level; 0 under the other drivers) */
+    float* level_ms;
 } xbfs_run_stats;
 
 /* kernel ids reported in xbfs_run_stats.kernel_id */

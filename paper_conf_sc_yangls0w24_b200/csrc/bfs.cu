@@ -164,9 +164,8 @@ __device__ __forceinline__ void mirror_host(const KArgs& a, const DevState* st) 
 }
 
 // ---------------------------------------------------------------- init
-__global__ __launch_bounds__(256) void k_init_fill(KArgs a, int* __restrict__ level, int* __restrict__ parent,
-                                                   const unsigned int* __restrict__ nonisolated) {
-    count_launch(a.st);
+__device__ __forceinline__ void init_body(const KArgs& a, int* __restrict__ level, int* __restrict__ parent,
+                                          const unsigned int* __restrict__ nonisolated) {
     const long long tid = blockIdx.x * (long long)blockDim.x + threadIdx.x;
     const long long nth = (long long)gridDim.x * blockDim.x;
     const long long n4 = a.n / 4;
@@ -188,6 +187,12 @@ __global__ __launch_bounds__(256) void k_init_fill(KArgs a, int* __restrict__ le
     }
 }
 
+__global__ __launch_bounds__(256) void k_init_fill(KArgs a, int* __restrict__ level, int* __restrict__ parent,
+                                                   const unsigned int* __restrict__ nonisolated) {
+    count_launch(a.st);
+    init_body(a, level, parent, nonisolated);
+}
+
 __device__ int choose_strategy(const DevState* st, long long arcs, long long fsize, long long fprev,
                                long long fedges, long long unvisited, int prev) {
     if (st->force >= 0) return st->force;
@@ -201,15 +206,15 @@ __device__ int choose_strategy(const DevState* st, long long arcs, long long fsi
 }
 
 // Seed the source (the source holds level 0) and reset the level state.
-__global__ void k_seed(KArgs a, int* level, int* parent, long long nonisolated_count) {
-    count_launch(a.st);
+// One thread.
+__device__ __forceinline__ void seed_body(const KArgs& a, int* level, int* parent, long long nonisolated_count) {
     DevState* st = a.st;
     const long long s = st->source;   // per-run parameter copied in before init
     const long long rs = a.row_ptr[s], deg = a.row_ptr[s + 1] - rs;
     level[s] = 0;
     parent[s] = (int)s;
-    a.visited[s >> 5] |= 1u << (s & 31);
-    a.fb[0][s >> 5] |= 1u << (s & 31);
+    atomicOr(a.visited + (s >> 5), 1u << (s & 31));
+    atomicOr(a.fb[0] + (s >> 5), 1u << (s & 31));
     a.qv[0][0] = (int)s;
     a.qoff[0][0] = 0;
     a.qdelta[0][0] = rs;
@@ -232,71 +237,128 @@ __global__ void k_seed(KArgs a, int* level, int* parent, long long nonisolated_c
     st->fedges = deg;
     st->fprev = 0;
     st->unvisited = nonisolated_count - (deg > 0 ? 1 : 0);
-    st->acc_found = st->acc_edges = st->acc_probes = 0;
+    for (int i = 0; i < 3; ++i) st->acc_found[i] = st->acc_edges[i] = st->acc_probes[i] = 0;
     st->reached = 0;
     st->arcs_traversed = 0;
     st->nlevels = 0;
     st->source = s;
     st->prev_strategy = -1;
     st->strategy = choose_strategy(st, a.arcs, 1, 0, deg, st->unvisited, -1);
-    mirror_host(a, st);
+}
+
+__global__ void k_seed(KArgs a, int* level, int* parent, long long nonisolated_count) {
+    count_launch(a.st);
+    seed_body(a, level, parent, nonisolated_count);
+    mirror_host(a, a.st);
 }
 
 // ------------------------------------------------------------- select
-// End of level k: consolidate the counters, log the level, choose the strategy of
-// level k+1 (P:L87 rule + readings C-10/C-11) and rotate the counter slots.
-// One thread (k_select).  Fusing it into the last block of the level kernels was
-// measured slower: it raised their register pressure (spills).
-__device__ void select_body(const KArgs& a) {
-    // one parallel read of the whole state (independent loads in flight together),
-    // then plain stores: the selector is on the critical path of every level
-    DevState local = *a.st;
-    DevState* st = &local;
-    const int k = st->k;
-    const int strat = st->strategy;
+// The level state the selector evolves (one copy per CTA in the persistent
+// driver, where every CTA computes the same decision from the same counters).
+struct SelState {
+    int k, strategy, queue_valid, done, prev_strategy, nlevels, prev_small, pad_;
+    long long fsize, fedges, fprev, unvisited, reached, arcs_traversed;
+    unsigned fmaxdeg;
+};
+
+// End of level k: consolidate the counters of F_{k+1} (acc slot k%3 after BU / SS,
+// queue counter (k+1)%3 after SF), log the level (if `log_it`), choose the
+// strategy of level k+1 (P:L87 rule + readings C-10/C-11).  All counter reads go
+// through L2.
+__device__ __forceinline__ void select_step(const KArgs& a, SelState& s, bool log_it, unsigned long long t_ns) {
+    const DevState* st = a.st;
+    const int k = s.k;
+    const int strat = s.strategy;
     long long nf, ne;
     if (strat == XBFS_BU || strat == XBFS_SS) {   // counted by k_bu_traverse / k_ss_count; no queue
-        nf = (long long)st->acc_found;
-        ne = (long long)st->acc_edges;
-        st->queue_valid = 0;
+        nf = (long long)__ldcg(&st->acc_found[k % 3]);
+        ne = (long long)__ldcg(&st->acc_edges[k % 3]);
+        s.queue_valid = 0;
     } else {
-        const unsigned long long q = st->qctr[(k + 1) % 3];
+        const unsigned long long q = __ldcg(&st->qctr[(k + 1) % 3]);
         nf = (long long)(q >> a.dbits);
         ne = (long long)(q & ((1ull << a.dbits) - 1ull));
-        st->queue_valid = 1;
+        s.queue_valid = 1;
     }
-    if (k < kLogCap) {
+    if (log_it && k < kLogCap) {
         LevelRec r;
-        r.fsize = st->fsize;
-        r.fedges = st->fedges;
-        r.unvisited = st->unvisited;
-        r.probes = strat == XBFS_BU ? (long long)st->acc_probes : 0;
+        r.fsize = s.fsize;
+        r.fedges = s.fedges;
+        r.unvisited = s.unvisited;
+        r.probes = strat == XBFS_BU ? (long long)__ldcg(&st->acc_probes[k % 3]) : 0;
         r.strategy = strat;
         r.pad = 0;
+        r.t_ns = t_ns;
         a.log[k] = r;
     }
     // enter the small-frontier mode only after one small SF level has already run
     // through the level kernels (a single small level does not pay for the switch)
-    st->prev_small = strat == XBFS_SF && st->fedges <= st->small_edges && st->fmaxdeg <= (unsigned)kSmallMaxDeg;
-    st->reached += st->fsize;
-    st->arcs_traversed += st->fedges;
-    st->fprev = st->fsize;
-    st->fsize = nf;
-    st->fedges = ne;
-    st->unvisited -= nf;
-    st->acc_found = st->acc_edges = st->acc_probes = 0;
-    st->prev_strategy = strat;
-    st->k = k + 1;
-    st->fmaxdeg = st->qmax[(k + 1) % 3];
+    s.prev_small = strat == XBFS_SF && s.fedges <= st->small_edges && s.fmaxdeg <= (unsigned)kSmallMaxDeg;
+    s.reached += s.fsize;
+    s.arcs_traversed += s.fedges;
+    s.fprev = s.fsize;
+    s.fsize = nf;
+    s.fedges = ne;
+    s.unvisited -= nf;
+    s.prev_strategy = strat;
+    s.k = k + 1;
+    s.fmaxdeg = __ldcg(&st->qmax[(k + 1) % 3]);
+    if (nf == 0) {
+        s.done = 1;
+        s.nlevels = k + 1;
+    } else {
+        s.strategy = choose_strategy(st, a.arcs, nf, s.fprev, ne, s.unvisited, strat);
+    }
+}
+
+__device__ __forceinline__ void sel_load(const DevState* st, SelState& s) {
+    s.k = __ldcg(&st->k);
+    s.strategy = __ldcg(&st->strategy);
+    s.queue_valid = __ldcg(&st->queue_valid);
+    s.done = __ldcg(&st->done);
+    s.prev_strategy = __ldcg(&st->prev_strategy);
+    s.nlevels = __ldcg(&st->nlevels);
+    s.prev_small = __ldcg(&st->prev_small);
+    s.fsize = __ldcg(&st->fsize);
+    s.fedges = __ldcg(&st->fedges);
+    s.fprev = __ldcg(&st->fprev);
+    s.unvisited = __ldcg(&st->unvisited);
+    s.reached = __ldcg(&st->reached);
+    s.arcs_traversed = __ldcg(&st->arcs_traversed);
+    s.fmaxdeg = __ldcg(&st->fmaxdeg);
+}
+
+__device__ __forceinline__ void sel_store(DevState* st, const SelState& s) {
+    st->k = s.k;
+    st->strategy = s.strategy;
+    st->queue_valid = s.queue_valid;
+    st->done = s.done;
+    st->prev_strategy = s.prev_strategy;
+    st->nlevels = s.nlevels;
+    st->prev_small = s.prev_small;
+    st->fsize = s.fsize;
+    st->fedges = s.fedges;
+    st->fprev = s.fprev;
+    st->unvisited = s.unvisited;
+    st->reached = s.reached;
+    st->arcs_traversed = s.arcs_traversed;
+    st->fmaxdeg = s.fmaxdeg;
+}
+
+// Per-level kernels: one thread reads the state, steps it, writes it back and
+// zeroes the slots level k+1 accumulates into (qctr/qmax (k+2)%3, acc (k+1)%3).
+// Fusing it into the last block of the level kernels was measured slower: it
+// raised their register pressure (spills).
+__device__ void select_body(const KArgs& a) {
+    DevState* st = a.st;
+    SelState s;
+    sel_load(st, s);
+    const int k = s.k;
+    select_step(a, s, true, 0ull);
     st->qctr[(k + 2) % 3] = 0;   // counter of the queue built during level k+1
     st->qmax[(k + 2) % 3] = 0;
-    if (nf == 0) {
-        st->done = 1;
-        st->nlevels = k + 1;
-    } else {
-        st->strategy = choose_strategy(st, a.arcs, nf, st->fprev, ne, st->unvisited, strat);
-    }
-    *a.st = local;
+    st->acc_found[(k + 1) % 3] = st->acc_edges[(k + 1) % 3] = st->acc_probes[(k + 1) % 3] = 0;
+    sel_store(st, s);
     mirror_host(a, st);
 }
 
@@ -305,14 +367,18 @@ __device__ void select_body(const KArgs& a) {
 // entry overlapping it, so tiles are balanced regardless of the degree mix
 // (hubs span many tiles, small vertices share one).  Arc a of the frontier is
 // col[a + qdelta[j]] for its owner j (binary search of qoff in shared memory).
-template <int MODE>
-__global__ __launch_bounds__(kExpandThreads, 3) void k_td_expand(KArgs a, int* __restrict__ level,
-                                                                int* __restrict__ parent) {
-    count_launch(a.st);
-    const int k = a.st->k;
+struct TdSmem {
+    long long off[kTile + 1];
+    long long delta[kTile + 1];
+    int v[kTile + 1];
+};
+
+template <int MODE, int THREADS>
+__device__ __forceinline__ void td_expand_body(const KArgs& a, int k, int* __restrict__ level,
+                                               int* __restrict__ parent, TdSmem& sm) {
     clear_stale(a, k);
     const int in = k % 3, ob = (k + 1) % 3;
-    const unsigned long long q = a.st->qctr[k % 3];
+    const unsigned long long q = __ldcg(&a.st->qctr[k % 3]);
     const long long F = (long long)(q >> a.dbits);
     const long long T = (long long)(q & ((1ull << a.dbits) - 1ull));
     if (F == 0 || T == 0) return;
@@ -324,35 +390,34 @@ __global__ __launch_bounds__(kExpandThreads, 3) void k_td_expand(KArgs a, int* _
     unsigned int* __restrict__ visited = a.visited;
     unsigned int* __restrict__ next = a.fb[(k + 1) % 3];
     const int lvl = k + 1;
-
-    __shared__ long long s_off[kTile + 1];
-    __shared__ long long s_delta[kTile + 1];
-    __shared__ int s_v[kTile + 1];
+    long long* s_off = sm.off;
+    long long* s_delta = sm.delta;
+    int* s_v = sm.v;
     unsigned lmax = 0;
 
     for (long long t = blockIdx.x; t < ntiles; t += gridDim.x) {
         const long long a0 = t * kTile;
         const long long a1 = min(a0 + (long long)kTile, T);
-        const long long i0 = tfirst[t];
-        const long long i1 = (t + 1 < ntiles) ? (long long)tfirst[t + 1] : F - 1;
+        const long long i0 = __ldcg(tfirst + t);
+        const long long i1 = (t + 1 < ntiles) ? (long long)__ldcg(tfirst + t + 1) : F - 1;
         const int nv = (int)(i1 - i0 + 1);
         __syncthreads();
-        for (int i = threadIdx.x; i < nv; i += blockDim.x) {
-            s_off[i] = qoff[i0 + i];
-            s_delta[i] = qdelta[i0 + i];
-            s_v[i] = qv[i0 + i];
+        for (int i = threadIdx.x; i < nv; i += THREADS) {
+            s_off[i] = __ldcg(qoff + i0 + i);
+            s_delta[i] = __ldcg(qdelta + i0 + i);
+            s_v[i] = __ldcg(qv + i0 + i);
         }
         __syncthreads();
-        // R arcs per thread (stride blockDim: coalesced col reads), processed
+        // R arcs per thread (stride THREADS: coalesced col reads), processed
         // stage by stage so the R dependent load chains are in flight together.
-        constexpr int R = kTile / kExpandThreads;
+        constexpr int R = kTile / THREADS;
         int v[R], u[R];
         unsigned vis[R];
         bool valid[R], win[R];
         long long rs[R], deg[R];
 #pragma unroll
         for (int i = 0; i < R; ++i) {
-            const long long arc = a0 + i * kExpandThreads + threadIdx.x;
+            const long long arc = a0 + i * THREADS + threadIdx.x;
             valid[i] = arc < a1;
             v[i] = 0;
             u[i] = 0;
@@ -414,26 +479,28 @@ __global__ __launch_bounds__(kExpandThreads, 3) void k_td_expand(KArgs a, int* _
     if (MODE == XBFS_SF) flush_max(&a.st->qmax[(k + 1) % 3], lmax);
 }
 
+template <int MODE>
+__global__ __launch_bounds__(kExpandThreads, 3) void k_td_expand(KArgs a, int* __restrict__ level,
+                                                                int* __restrict__ parent) {
+    count_launch(a.st);
+    __shared__ TdSmem sm;
+    td_expand_body<MODE, kExpandThreads>(a, a.st->k, level, parent, sm);
+}
+
 // -------------------------------------------------------------- generate
-// Bitmap -> queue (the single-scan generation pass, over the N-bit frontier
-// bitmap instead of the 4N-byte status array).  role 0: F_k from fb[k%3] into
-// queue k&1 (queue missing after a BU level).  role 1: F_{k+1} from
-// fb[(k+1)%3] into queue (k+1)&1 and visited |= F_{k+1} (after SS expansion).
 // Single-scan's one scan over the status, here the N-bit next-frontier
 // bitmap: it yields the counters the selector needs (|F_{k+1}|, edgesF_{k+1},
-// max degree, from the dense head[] array).  The queue itself is materialised by
-// k_generate(role 0) only if the next level is top-down; a bottom-up next level
-// never needs it (the bitmap is its input).  visited already holds F_{k+1}: the
-// expansion set it with REDs.
-__global__ __launch_bounds__(kGenThreads) void k_ss_count(KArgs a) {
-    count_launch(a.st);
-    const int k = a.st->k;
+// max degree, from the dense head[] array) into acc slot k%3.  The queue itself
+// is materialised by generate (role 0) only if the next level is top-down; a
+// bottom-up next level never needs it (the bitmap is its input).  visited
+// already holds F_{k+1}: the expansion set it with REDs.
+__device__ __forceinline__ void ss_count_body(const KArgs& a, int k) {
     const unsigned int* __restrict__ bm = a.fb[(k + 1) % 3];
     unsigned long long found = 0, edges = 0;
     unsigned gmax = 0;
     for (long long w = blockIdx.x * (long long)blockDim.x + threadIdx.x; w < a.words;
          w += (long long)gridDim.x * blockDim.x) {
-        const unsigned word = bm[w];
+        const unsigned word = __ldcg(bm + w);
         if (!word) continue;
         found += __popc(word);
         for (unsigned b = word; b; b &= b - 1) {
@@ -448,15 +515,22 @@ __global__ __launch_bounds__(kGenThreads) void k_ss_count(KArgs a) {
         edges += __shfl_xor_sync(FULL, edges, o);
     }
     if ((threadIdx.x & 31) == 0 && found) {
-        atomicAdd(&a.st->acc_found, found);
-        atomicAdd(&a.st->acc_edges, edges);
+        atomicAdd(&a.st->acc_found[k % 3], found);
+        atomicAdd(&a.st->acc_edges[k % 3], edges);
     }
     flush_max(&a.st->qmax[(k + 1) % 3], gmax);
 }
 
-__global__ __launch_bounds__(kGenThreads) void k_generate(KArgs a, int role) {
+__global__ __launch_bounds__(kGenThreads) void k_ss_count(KArgs a) {
     count_launch(a.st);
-    const int k = a.st->k;
+    ss_count_body(a, a.st->k);
+}
+
+// Bitmap -> queue (the single-scan generation pass, over the N-bit frontier
+// bitmap instead of the 4N-byte status array).  role 0: F_k from fb[k%3] into
+// queue slot k%3 (queue missing after a BU / SS level).  role 1: F_{k+1} from
+// fb[(k+1)%3] into slot (k+1)%3 and visited |= F_{k+1}.
+__device__ __forceinline__ void generate_body(const KArgs& a, int k, int role) {
     const unsigned int* __restrict__ bm = role == 0 ? a.fb[k % 3] : a.fb[(k + 1) % 3];
     const int ob = role == 0 ? k % 3 : (k + 1) % 3;
     unsigned long long* ctr = &a.st->qctr[role == 0 ? k % 3 : (k + 1) % 3];
@@ -466,8 +540,8 @@ __global__ __launch_bounds__(kGenThreads) void k_generate(KArgs a, int role) {
     unsigned gmax = 0;
     for (long long w0 = base_tid; w0 < a.words; w0 += nth) {
         const long long w = w0 + lane;
-        unsigned word = w < a.words ? bm[w] : 0u;
-        if (role == 1 && word) a.visited[w] |= word;
+        unsigned word = w < a.words ? __ldcg(bm + w) : 0u;
+        if (role == 1 && word) a.visited[w] = __ldcg(a.visited + w) | word;
         // pass 1: count and degree sum of this lane's vertices
         const int cnt = __popc(word);
         long long dsum = 0;
@@ -514,14 +588,22 @@ __global__ __launch_bounds__(kGenThreads) void k_generate(KArgs a, int role) {
     flush_max(&a.st->qmax[role == 0 ? k % 3 : (k + 1) % 3], gmax);
 }
 
+__global__ __launch_bounds__(kGenThreads) void k_generate(KArgs a, int role) {
+    count_launch(a.st);
+    generate_body(a, a.st->k, role);
+}
+
 // ------------------------------------------------------------- bottom-up
 // Candidates U_k = not visited (isolated vertices are pre-marked visited).
 // A candidate v is found iff some neighbour is in F_k = fb[k%3] (never a bit set
 // in this same pass: reading C-9), giving level k+1 and that neighbour as parent.
-__global__ __launch_bounds__(kBuThreads, 5) void k_bu_traverse(KArgs a, int* __restrict__ level,
-                                                            int* __restrict__ parent) {
-    count_launch(a.st);
-    const int k = a.st->k;
+// kp: where k lives (DevState or the persistent CTA's selector copy); it is
+// re-read for the epilogue instead of keeping k live across the traversal
+// (one register less: the per-level kernel runs at 48 without spills).
+template <int WARPS>
+__device__ __forceinline__ void bu_body(const KArgs& a, const int* kp, int* __restrict__ level,
+                                        int* __restrict__ parent, BuSmem<WARPS>& sm) {
+    int k = *(const volatile int*)kp;
     clear_stale(a, k);
     const unsigned int* __restrict__ cur = a.fb[k % 3];
     unsigned int* __restrict__ next = a.fb[(k + 1) % 3];
@@ -538,7 +620,7 @@ __global__ __launch_bounds__(kBuThreads, 5) void k_bu_traverse(KArgs a, int* __r
     b.level = level;
     b.parent = parent;
     b.lvl = lvl;
-    bu_chunks(b, [&](long long w, unsigned vis, unsigned f) {
+    bu_chunks<WARPS>(b, sm, [&](long long w, unsigned vis, unsigned f) {
         next[w] = f;
         if (f) a.visited[w] = vis | f;
     }, found, edges, probes, fmax);
@@ -549,15 +631,23 @@ __global__ __launch_bounds__(kBuThreads, 5) void k_bu_traverse(KArgs a, int* __r
         edges += __shfl_xor_sync(FULL, edges, o);
         probes += __shfl_xor_sync(FULL, probes, o);
     }
+    k = *(const volatile int*)kp;
     if (lane == 0 && (found | edges | probes)) {
-        atomicAdd(&a.st->acc_found, found);
-        atomicAdd(&a.st->acc_edges, edges);
-        atomicAdd(&a.st->acc_probes, probes);
+        atomicAdd(&a.st->acc_found[k % 3], found);
+        atomicAdd(&a.st->acc_edges[k % 3], edges);
+        atomicAdd(&a.st->acc_probes[k % 3], probes);
     }
     fmax = __reduce_max_sync(FULL, fmax);
     if (lane == 0 && fmax) {
         atomic_max_if_greater(&a.st->qmax[(k + 1) % 3], fmax);
     }
+}
+
+__global__ __launch_bounds__(kBuThreads, 5) void k_bu_traverse(KArgs a, int* __restrict__ level,
+                                                            int* __restrict__ parent) {
+    count_launch(a.st);
+    __shared__ BuSmem<kBuThreads / 32> sm;
+    bu_body<kBuThreads / 32>(a, &a.st->k, level, parent, sm);
 }
 
 // ---------------------------------------------------------------- select
@@ -757,7 +847,7 @@ __global__ void __cluster_dims__(kSmallCluster, 1, 1) __launch_bounds__(kSmallTh
         st->reached = reached;
         st->arcs_traversed = arcs_tr;
         st->prev_strategy = XBFS_SF;
-        st->acc_found = st->acc_edges = st->acc_probes = 0;
+        for (int i = 0; i < 3; ++i) st->acc_found[i] = st->acc_edges[i] = st->acc_probes[i] = 0;
         st->fmaxdeg = fmaxdeg;
         st->advanced = st->mirror_host ? 0 : 1;   // graph driver: its k_select node only mirrors
         st->prev_small = 1;
@@ -774,6 +864,101 @@ __global__ __launch_bounds__(256) void k_count_m(const int* __restrict__ level, 
         if (level[v] >= 0) s += (unsigned long long)tcount[v];
     for (int o = 16; o; o >>= 1) s += __shfl_xor_sync(FULL, s, o);
     if ((threadIdx.x & 31) == 0 && s) atomicAdd(out, s);
+}
+
+// ------------------------------------------------- persistent driver
+// One cooperative launch per BFS: init, seed and every level run inside one
+// kernel whose CTAs are all co-resident (cudaLaunchCooperativeKernel checks it),
+// separated by grid barriers instead of kernel boundaries.  The level loop's
+// fixed cost (~20 us per level through launches + a 1-thread select kernel, both
+// for the host loop and the CUDA-graph loop, tools/level_floor.py) becomes one
+// or two grid barriers.  Every CTA steps its own copy of the selector state from
+// the same counters (deterministic), so the decision needs no extra barrier;
+// CTA 0 also logs the level and its %globaltimer stamp.
+__device__ __forceinline__ unsigned long long globaltimer() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+
+__device__ __forceinline__ unsigned ld_acquire(const unsigned* p) {
+    unsigned v;
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+
+// Grid barrier: monotonic arrival counter (zeroed with the state before the
+// run); barrier e completes when it reaches e * gridDim.x.  __syncthreads +
+// the release fence before the arrival and the acquire load after it order
+// every write of the phase before every read of the next (mutable state is
+// read through L2 everywhere).  A barrier that does not complete within 10 s
+// traps: the run fails with a CUDA error (handle poisoned) instead of hanging.
+__device__ __forceinline__ void grid_sync(unsigned* ctr, unsigned& epoch) {
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        ++epoch;
+        const unsigned target = epoch * gridDim.x;
+        __threadfence();
+        atomicAdd(ctr, 1u);
+        if ((int)(ld_acquire(ctr) - target) < 0) {
+            const unsigned long long t0 = globaltimer();
+            while ((int)(ld_acquire(ctr) - target) < 0)
+                if (globaltimer() - t0 > 10000000000ull) __trap();
+        }
+    }
+    __syncthreads();
+}
+
+union PersistSmem {
+    TdSmem td;
+    BuSmem<kPersistThreads / 32> bu;
+};
+
+__global__ __launch_bounds__(kPersistThreads, kPersistBlocks) void k_persist(
+    KArgs a, int* __restrict__ level, int* __restrict__ parent, const unsigned int* __restrict__ nonisolated,
+    long long nonisolated_count) {
+    extern __shared__ __align__(16) unsigned char dsm[];
+    PersistSmem& sm = *reinterpret_cast<PersistSmem*>(dsm);
+    __shared__ SelState s;
+    unsigned epoch = 0;
+    unsigned* bar = &a.st->bar_count;
+    count_launch(a.st);
+    init_body(a, level, parent, nonisolated);
+    grid_sync(bar, epoch);
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        seed_body(a, level, parent, nonisolated_count);
+        a.st->t_start = globaltimer();
+    }
+    grid_sync(bar, epoch);
+    if (threadIdx.x == 0) sel_load(a.st, s);
+    __syncthreads();
+    for (;;) {
+        const int k = s.k, strat = s.strategy, qvalid = s.queue_valid;
+        if (s.done) break;
+        if (blockIdx.x == 0 && threadIdx.x == 0) {
+            // slots nobody touches during level k (see select_body)
+            a.st->qctr[(k + 2) % 3] = 0;
+            a.st->qmax[(k + 2) % 3] = 0;
+            a.st->acc_found[(k + 1) % 3] = a.st->acc_edges[(k + 1) % 3] = a.st->acc_probes[(k + 1) % 3] = 0;
+        }
+        if (strat != XBFS_BU && !qvalid) {
+            generate_body(a, k, 0);
+            grid_sync(bar, epoch);
+        }
+        if (strat == XBFS_SF) {
+            td_expand_body<XBFS_SF, kPersistThreads>(a, k, level, parent, sm.td);
+        } else if (strat == XBFS_SS) {
+            td_expand_body<XBFS_SS, kPersistThreads>(a, k, level, parent, sm.td);
+            grid_sync(bar, epoch);
+            ss_count_body(a, k);
+        } else {
+            bu_body<kPersistThreads / 32>(a, &s.k, level, parent, sm.bu);
+        }
+        grid_sync(bar, epoch);
+        if (threadIdx.x == 0) select_step(a, s, blockIdx.x == 0, blockIdx.x == 0 ? globaltimer() : 0ull);
+        __syncthreads();
+    }
+    if (blockIdx.x == 0 && threadIdx.x == 0) sel_store(a.st, s);
 }
 
 // ------------------------------------------------------------- drivers
@@ -1021,6 +1206,30 @@ xbfs_status build_loop_graph(xbfs_graph* g, int* level, int* parent) {
     return XBFS_OK;
 }
 
+xbfs_status launch_persist(xbfs_graph* g, const KArgs& a, int* level, int* parent) {
+    static int occ[64];
+    static bool init[64] = {false};
+    const int dev = g->device & 63;
+    if (!init[dev]) {
+        XBFS_CUDA(g, cudaFuncSetAttribute(k_persist, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                          (int)sizeof(PersistSmem)));
+        int o = 0;
+        XBFS_CUDA(g, cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, k_persist, kPersistThreads,
+                                                                   sizeof(PersistSmem)));
+        occ[dev] = o;
+        init[dev] = true;
+    }
+    if (occ[dev] < 1) return set_error(XBFS_ERR_UNSUPPORTED, "persistent driver: k_persist does not fit on an SM");
+    const int grid = g->num_sms * std::min(occ[dev], kPersistBlocks);
+    const unsigned int* noniso = g->nonisolated;
+    long long nic = g->nonisolated_count;
+    KArgs ka = a;
+    void* args[] = {&ka, &level, &parent, &noniso, &nic};
+    XBFS_CUDA(g, cudaLaunchCooperativeKernel((void*)k_persist, dim3(grid), dim3(kPersistThreads), args,
+                                             sizeof(PersistSmem), g->stream));
+    return XBFS_OK;
+}
+
 }  // namespace
 }  // namespace xbfs
 
@@ -1041,8 +1250,10 @@ static xbfs_status run_impl(xbfs_graph* g, int64_t source, int32_t* level, int32
     XBFS_CUDA(g, cudaSetDevice(g->device));
 
     KArgs a = g->kargs();
-    const bool use_graph = (o.driver == 0 || o.driver == 2) && !(stats && stats->kernel_capacity > 0) &&
-                           !(o.plan && o.plan_len > 0);
+    if (o.driver < 0 || o.driver > 3) return set_error(XBFS_ERR_INVALID_ARG, "driver must be 0..3");
+    const bool host_only = (stats && stats->kernel_capacity > 0) || (o.plan && o.plan_len > 0);
+    const bool use_persist = (o.driver == 0 || o.driver == 3) && !host_only;
+    const bool use_graph = o.driver == 2 && !host_only;
     // selection parameters live in the device state
     {
         DevState hs;
@@ -1054,14 +1265,18 @@ static xbfs_status run_impl(xbfs_graph* g, int64_t source, int32_t* level, int32
         hs.force = o.force_strategy;
         hs.source = source;
         hs.small_edges = std::min<long long>(std::max(o.small_edges, 0), kSmallEdgesMax);
-        hs.mirror_host = use_graph ? 0 : 1;
+        hs.mirror_host = (use_graph || use_persist) ? 0 : 1;
         XBFS_CUDA(g, cudaMemcpyAsync(g->st, &hs, sizeof(hs), cudaMemcpyHostToDevice, g->stream));
     }
     const Grids G = grids_for(g);
     Prof P;
     P.g = g;
     P.st = stats;
-    if (use_graph) {
+    if (use_persist) {
+        XBFS_CUDA(g, cudaEventRecord(g->ev0, g->stream));
+        XBFS_TRY(launch_persist(g, a, level, parent));
+        XBFS_CUDA(g, cudaEventRecord(g->ev1, g->stream));
+    } else if (use_graph) {
         XBFS_TRY(build_loop_graph(g, level, parent));
         XBFS_CUDA(g, cudaEventRecord(g->ev0, g->stream));
         XBFS_CUDA(g, cudaGraphLaunch(g->cur_exec, g->stream));
@@ -1097,7 +1312,7 @@ static xbfs_status run_impl(xbfs_graph* g, int64_t source, int32_t* level, int32
         XBFS_TRY(P.finish());
         const int nl = std::min(hs.nlevels, std::min(stats->level_capacity, kLogCap));
         if (nl > 0 && (stats->strategy || stats->frontier_vertices || stats->frontier_edges ||
-                       stats->unvisited || stats->bu_probes)) {
+                       stats->unvisited || stats->bu_probes || stats->level_ms)) {
             LevelRec* rec = new LevelRec[nl];
             XBFS_CUDA(g, cudaMemcpy(rec, g->log, nl * sizeof(LevelRec), cudaMemcpyDeviceToHost));
             for (int i = 0; i < nl; ++i) {
@@ -1106,6 +1321,11 @@ static xbfs_status run_impl(xbfs_graph* g, int64_t source, int32_t* level, int32
                 if (stats->frontier_edges) stats->frontier_edges[i] = rec[i].fedges;
                 if (stats->unvisited) stats->unvisited[i] = rec[i].unvisited;
                 if (stats->bu_probes) stats->bu_probes[i] = rec[i].probes;
+                if (stats->level_ms) {
+                    const unsigned long long t0 = i ? rec[i - 1].t_ns : hs.t_start;
+                    stats->level_ms[i] = (use_persist && rec[i].t_ns >= t0 && t0) ? (float)((rec[i].t_ns - t0) * 1e-6)
+                                                                                   : 0.f;
+                }
             }
             delete[] rec;
         }

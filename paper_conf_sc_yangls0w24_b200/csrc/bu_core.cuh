@@ -20,18 +20,31 @@ struct BuView {
     int lvl;                          // k + 1
 };
 
+// Per-warp shared-memory work lists of one block of WARPS warps (static in the
+// per-level kernels, carved from dynamic shared memory in the persistent one).
+template <int WARPS>
+struct BuSmem {
+    int list[WARPS][kBuChunkWords * 32];   // candidates of the warp's chunk
+    int hard[WARPS][kBuChunkWords * 32];   // long unresolved rows (warp-cooperative)
+    int hoff[WARPS][kBuChunkWords * 32];   // arcs already probed for each hard row
+    unsigned found[WARPS][kBuChunkWords];
+};
+
 // publish(w, vis, found_word): store the owned word w of F_{k+1} and update visited.
-template <class Publish>
-__device__ __forceinline__ void bu_chunks(const BuView& b, Publish publish, unsigned long long& found,
-                                          unsigned long long& edges, unsigned long long& probes, unsigned& fmax) {
+// Mutable state (visited, cur) is read through L2 (__ldcg): the persistent
+// driver runs every level inside one kernel, where L1 lines are not refreshed.
+template <int WARPS, class Publish>
+__device__ __forceinline__ void bu_chunks(const BuView& b, BuSmem<WARPS>& sm, Publish publish,
+                                          unsigned long long& found, unsigned long long& edges,
+                                          unsigned long long& probes, unsigned& fmax) {
     constexpr unsigned FULL = 0xffffffffu;
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
     const unsigned lt = (1u << lane) - 1u;
-    constexpr int kCW = kBuChunkWords, kCV = kBuChunkWords * 32;
-    __shared__ int s_list[kBuThreads / 32][kCV];   // candidates of the warp's chunk
-    __shared__ int s_hard[kBuThreads / 32][kCV];   // long unresolved rows (warp-cooperative)
-    __shared__ int s_hoff[kBuThreads / 32][kCV];   // arcs already probed for each hard row
-    __shared__ unsigned s_found[kBuThreads / 32][kCW];
+    constexpr int kCW = kBuChunkWords;
+    auto& s_list = sm.list;
+    auto& s_hard = sm.hard;
+    auto& s_hoff = sm.hoff;
+    auto& s_found = sm.found;
     const long long nchunks = (b.words + kCW - 1) / kCW;
     const long long gw = (blockIdx.x * (long long)blockDim.x + threadIdx.x) >> 5;
     const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
@@ -40,7 +53,7 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, Publish publish, unsi
         //    (the paper's count + prefix-sum + queue-write "double scan").
         const long long w = c * kCW + lane;
         const bool own = lane < kCW && w < b.words;
-        const unsigned vis = own ? b.visited[w] : FULL;
+        const unsigned vis = own ? __ldcg(b.visited + w) : FULL;
         const unsigned cand = ~vis;
         // fast path: no candidate in the chunk (most chunks in late BU levels); F_{k+1}
         // words start out zero (the stale-bitmap clear of level k-1), so nothing to write

@@ -38,10 +38,13 @@ constexpr int kSmallBig = 8192;      // per-CTA list of higher-degree vertices (
 constexpr long long kSmallEdgesMax = 9LL * kSmallBig;  // guarantees the big list never overflows
 constexpr int kSmallMaxDeg = 512;    // frontier max degree allowed in the small mode (warp steps <= 16)
 constexpr int kLogCap = 1 << 16;     // per-level log entries kept on the device
+constexpr int kPersistThreads = 512; // persistent (one launch per BFS) driver: threads per CTA
+constexpr int kPersistBlocks = 2;    // ... CTAs per SM (64 registers per thread)
 
 struct LevelRec {
     long long fsize, fedges, unvisited, probes;
     int strategy, pad;
+    unsigned long long t_ns;   // %globaltimer at the end of the level (persistent driver; 0 otherwise)
 };
 
 // Mirror of the scalars the host loop needs after each select (pinned + mapped).
@@ -64,7 +67,8 @@ struct DevState {
     long long fsize, fedges;     // |F_k|, edgesF_k
     long long fprev;             // |F_{k-1}|
     long long unvisited;         // U_k (non-isolated, unvisited)
-    unsigned long long acc_found, acc_edges, acc_probes;  // BU accumulators for level k
+    unsigned long long acc_found[3], acc_edges[3], acc_probes[3];  // BU / SS-count accumulators:
+                                 // level k adds into slot k%3; slot (k+1)%3 is zeroed before level k+1
     long long reached, arcs_traversed;
     unsigned int launches;       // library kernels launched (device-counted)
     int nlevels;
@@ -77,6 +81,11 @@ struct DevState {
     int prev_small;              // level k-1 was a small SF level (small-mode entry gate)
     int mirror_host;             // host-loop driver: mirror the level state into HostCtl
     int pad2_;
+    unsigned long long t_start;  // %globaltimer after init + seed (persistent driver)
+    // persistent driver: grid-barrier arrival counter, alone on its 128-byte line
+    // (zeroed with the rest of the state before every run)
+    alignas(128) unsigned bar_count;
+    unsigned bar_pad_[31];
 };
 
 // Arguments shared by all level kernels (static per handle => graph-capturable).

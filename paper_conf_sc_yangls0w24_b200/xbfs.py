@@ -55,7 +55,7 @@ class RunStats(ctypes.Structure):
                 ("bu_probes", ctypes.POINTER(ctypes.c_int64)),
                 ("kernel_capacity", ctypes.c_int32), ("num_kernels", ctypes.c_int32),
                 ("kernel_id", ctypes.POINTER(ctypes.c_int32)), ("kernel_level", ctypes.POINTER(ctypes.c_int32)),
-                ("kernel_ms", ctypes.POINTER(ctypes.c_float))]
+                ("kernel_ms", ctypes.POINTER(ctypes.c_float)), ("level_ms", ctypes.POINTER(ctypes.c_float))]
 
 
 #: kernel ids of RunStats.kernel_id (XBFS_K_* in include/xbfs.h)
@@ -174,6 +174,7 @@ class Stats:
     unvisited: list = field(default_factory=list)
     bu_probes: list = field(default_factory=list)
     kernels: list = field(default_factory=list)   # (name, level, ms) when profiled
+    level_ms: list = field(default_factory=list)  # device ms per level (persistent driver)
 
 
 class _StatsBuf:
@@ -184,6 +185,7 @@ class _StatsBuf:
         self.fe = np.zeros(cap, np.int64)
         self.un = np.zeros(cap, np.int64)
         self.pr = np.zeros(cap, np.int64)
+        self.lms = np.zeros(cap, np.float32)
         self.c = RunStats()
         self.c.level_capacity = cap
         P = lambda a, t: a.ctypes.data_as(ctypes.POINTER(t))
@@ -192,6 +194,7 @@ class _StatsBuf:
         self.c.frontier_edges = P(self.fe, ctypes.c_int64)
         self.c.unvisited = P(self.un, ctypes.c_int64)
         self.c.bu_probes = P(self.pr, ctypes.c_int64)
+        self.c.level_ms = P(self.lms, ctypes.c_float)
         self.kcap = kernel_cap
         if kernel_cap:
             self.kid = np.zeros(kernel_cap, np.int32)
@@ -209,7 +212,8 @@ class _StatsBuf:
                      c.kernel_launches, self.strategy[:nl].tolist(), self.fv[:nl].tolist(), self.fe[:nl].tolist(),
                      self.un[:nl].tolist(), self.pr[:nl].tolist(),
                      [(KERNEL_NAMES[int(self.kid[i])], int(self.klv[i]), float(self.kms[i]))
-                      for i in range(min(c.num_kernels, self.kcap))] if self.kcap else [])
+                      for i in range(min(c.num_kernels, self.kcap))] if self.kcap else [],
+                     self.lms[:nl].tolist())
 
 
 def make_run_opts(alpha=None, grow=None, ratio_min=None, bu_stay=None, force_strategy=None, driver=None,

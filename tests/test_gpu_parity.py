@@ -16,7 +16,9 @@ pytestmark = pytest.mark.gpu
 
 MODES = [dict(), dict(force_strategy=0), dict(force_strategy=1), dict(force_strategy=2),
          dict(alpha=0.02), dict(alpha=0.3, grow=1.0, ratio_min=0.0), dict(bu_stay=4.0),
-         dict(driver=1), dict(driver=1, force_strategy=1), dict(driver=1, force_strategy=2)]
+         dict(driver=1), dict(driver=1, force_strategy=1), dict(driver=1, force_strategy=2),
+         dict(driver=2), dict(driver=2, force_strategy=1), dict(driver=2, force_strategy=2),
+         dict(driver=3, force_strategy=0)]
 
 
 @pytest.fixture(scope="module")
@@ -233,6 +235,7 @@ def test_small_frontier_cluster_mode(xb, small):
         roots = [0, n - 1, n // 2] if graph == "grid" else synth.roots(n, src, dst, 5, root_seed=3)
         for root in roots:
             for opts in (dict(small_edges=small), dict(small_edges=small, driver=1),
+                         dict(small_edges=small, driver=2),
                          dict(small_edges=small, force_strategy=0), dict(small_edges=small, bu_stay=0.0)):
                 _check_run(g, og, src, dst, root, **opts)
         g.close()
@@ -252,4 +255,21 @@ def test_per_level_strategy_plan(xb):
             assert st.strategy == plan[:st.num_levels]
         st = _check_run(g, og, src, dst, root, plan=[-1, 2, -1])
         assert st.strategy[1] == 2
+    g.close()
+
+
+def test_persistent_driver_level_times(xb):
+    """The persistent driver (one cooperative launch per BFS) logs a %globaltimer
+    stamp per level: the per-level times are positive and sum to at most the
+    event-timed BFS; the other drivers report zeros."""
+    src, dst, n = synth.kronecker(16, seed=4)
+    og = oracle.build_csr(n, src, dst)
+    g = xb.Graph(_dev(src), _dev(dst), n)
+    for root in synth.roots(n, src, dst, 3, root_seed=5):
+        st = _check_run(g, og, src, dst, root, driver=3)
+        assert st.kernel_launches == 1
+        assert all(t > 0 for t in st.level_ms)
+        assert sum(st.level_ms) <= st.elapsed_ms * 1.01
+        st = _check_run(g, og, src, dst, root, driver=1)
+        assert st.kernel_launches > 1 and all(t == 0 for t in st.level_ms)
     g.close()
