@@ -99,6 +99,17 @@ def load_peaks():
         return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
 
 
+def load_traffic(cfg_name: str, kernel: str):
+    """DRAM bytes per launch (dram__bytes_read.sum + dram__bytes_write.sum) of
+    `kernel` from the committed `ncu --set full` capture of this bench command
+    (profiles/traffic.json, written by tools/ncu_traffic.py), or None."""
+    try:
+        d = json.load(open(os.path.join(ROOT, "profiles", "traffic.json")))
+        return d[workload_name(cfg_name)][kernel]["dram_bytes_per_launch"]
+    except Exception:
+        return None
+
+
 class ClockSampler:
     """nvidia-smi clocks + throttle reasons sampled during the timed region."""
 
@@ -232,12 +243,22 @@ def run_ours(args):
     torch.cuda.synchronize()
     per_root = []
     launches = 0
+    alg_bytes = 0
+    phase = {}          # strategy -> [levels, ms, algorithmic bytes] (persistent driver's level stamps)
     for r in mine:
         flush.fill_(1)                       # L2 flush, outside the timed region
         _, _, st = g.run(int(r), level, parent, stats=True, **opts)
         per_root.append((int(r), st.elapsed_ms, st.input_edges_traversed, st.arcs_traversed, st.num_levels,
                          "".join("FSB"[s] for s in st.strategy)))
         launches += st.kernel_launches
+        lb = metrics.bfs_level_bytes(n, st.strategy, st.frontier_vertices, st.frontier_edges, st.unvisited,
+                                     st.bu_probes)
+        alg_bytes += metrics.bytes_init(n) + sum(lb)
+        for s_, ms_, b_ in zip(st.strategy, st.level_ms, lb):
+            ph = phase.setdefault("FSB"[s_], [0, 0.0, 0])
+            ph[0] += 1
+            ph[1] += ms_
+            ph[2] += b_
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
@@ -289,13 +310,29 @@ def run_ours(args):
                    "bytes_per_launch": int(v[2] / v[0]),
                    "gbs": round(v[2] / (v[1] * 1e-3) / 1e9, 1) if v[1] > 0 else None}
                for k, v in agg.items()}
-    dom = max(agg.items(), key=lambda kv: kv[1][1])[0] if agg else None
     roofline = None
-    if dom:
+    timed_ms = sum(x[1] for x in per_root)
+    if launches == len(per_root):
+        # persistent driver: the timed region is ONE kernel launch per BFS (k_persist),
+        # so its event time per BFS is that kernel's launch duration
+        ach = alg_bytes / (timed_ms * 1e-3) / 1e9
+        bpl = int(alg_bytes / len(per_root))
+        roofline = {"bound": "hbm", "kernel": "k_persist", "achieved": round(ach, 1), "peak": peak, "unit": "GB/s",
+                    "frac": round(ach / peak, 4), "traffic": load_traffic(args.config, "k_persist"),
+                    "bytes_per_launch": bpl, "launch_ms": round(timed_ms / len(per_root), 4),
+                    "peak_source": peak_src,
+                    "phases": {k: {"levels": v[0], "ms": round(v[1], 4),
+                                   "gbs": round(v[2] / (v[1] * 1e-3) / 1e9, 1) if v[1] > 0 else None}
+                               for k, v in phase.items()},
+                    "note": "achieved = algorithmic bytes (init + every level, DESIGN.md §5) / event time of the "
+                            "single k_persist launch per BFS, over the timed roots; phases from the kernel's "
+                            "%globaltimer level stamps"}
+    elif agg:
+        dom = max(agg.items(), key=lambda kv: kv[1][1])[0]
         d = kernels[dom]
         ach = d["gbs"]
         roofline = {"bound": "hbm", "kernel": dom, "achieved": ach, "peak": peak, "unit": "GB/s",
-                    "frac": round(ach / peak, 4) if ach else None, "traffic": None,
+                    "frac": round(ach / peak, 4) if ach else None, "traffic": load_traffic(args.config, dom),
                     "bytes_per_launch": d["bytes_per_launch"], "peak_source": peak_src}
     b_model = metrics.model_bytes(n, g.arcs)
     model_frac = b_model / (ms_mean * 1e-3) / (peak * 1e9)
@@ -336,7 +373,9 @@ def run_ours(args):
         "config": {"workload": workload_name(args.config), "n_vertices": n, "input_edges": int(src.shape[0]),
                    "arcs": g.arcs, "roots_per_gpu": args.steps, "l2_flush": "512 MiB write before every timed BFS",
                    "reorder": "degree-desc (P:L153)", "alpha": opts.get("alpha", 0.1),
-                   "bu_stay": opts.get("bu_stay", 1.0), "driver": args.driver,
+                   "bu_stay": opts.get("bu_stay", 1.0),
+                   "driver": {0: "persistent (auto)", 1: "host loop", 2: "CUDA-graph loop",
+                              3: "persistent"}[args.driver],
                    "parallelism": f"replicas x{world} (independent roots)"},
         "gteps_hmean_per_gpu": round(worst["hmean"] / 1e9, 3),
         "gteps_arcs_hmean": round(res["teps_arcs"] / 1e9, 3),
@@ -429,7 +468,8 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--config", default="s24", choices=sorted(CONFIGS))
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--driver", type=int, default=1, help="0 auto, 1 host loop, 2 CUDA-graph device loop")
+    ap.add_argument("--driver", type=int, default=0,
+                    help="0 auto (= 3), 1 host loop, 2 CUDA-graph device loop, 3 persistent kernel")
     ap.add_argument("--alpha", type=float, default=None)
     ap.add_argument("--bu-stay", type=float, default=None)
     ap.add_argument("--small-edges", type=int, default=None)

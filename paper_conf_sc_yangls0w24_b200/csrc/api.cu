@@ -52,6 +52,7 @@ xbfs::KArgs xbfs_graph::kargs() const {
     a.words = words;
     a.arcs = arcs;
     a.dbits = dbits;
+    a.track_max = 1;
     return a;
 }
 

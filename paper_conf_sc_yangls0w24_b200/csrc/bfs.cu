@@ -58,6 +58,9 @@ __device__ __forceinline__ void atomic_max_if_greater(unsigned* p, unsigned v) {
     if (v > __ldcg(p)) atomicMax(p, v);
 }
 
+// Frontier max degree only gates the small-frontier cluster mode of the
+// per-level drivers; the persistent driver skips the tracking (KArgs.track_max).
+
 // Warp-reduce a per-lane max and publish it (call with the whole warp converged).
 __device__ __forceinline__ void flush_max(unsigned* p, unsigned lmax) {
     const unsigned w = __reduce_max_sync(FULL, lmax);
@@ -237,7 +240,7 @@ __device__ __forceinline__ void seed_body(const KArgs& a, int* level, int* paren
     st->fedges = deg;
     st->fprev = 0;
     st->unvisited = nonisolated_count - (deg > 0 ? 1 : 0);
-    for (int i = 0; i < 3; ++i) st->acc_found[i] = st->acc_edges[i] = st->acc_probes[i] = 0;
+    for (int i = 0; i < 3; ++i) st->acc_found[i] = st->acc_edges[i] = st->acc_probes[i] = st->grab[i] = 0;
     st->reached = 0;
     st->arcs_traversed = 0;
     st->nlevels = 0;
@@ -358,6 +361,7 @@ __device__ void select_body(const KArgs& a) {
     st->qctr[(k + 2) % 3] = 0;   // counter of the queue built during level k+1
     st->qmax[(k + 2) % 3] = 0;
     st->acc_found[(k + 1) % 3] = st->acc_edges[(k + 1) % 3] = st->acc_probes[(k + 1) % 3] = 0;
+    st->grab[(k + 1) % 3] = 0;
     sel_store(st, s);
     mirror_host(a, st);
 }
@@ -476,7 +480,7 @@ __device__ __forceinline__ void td_expand_body(const KArgs& a, int k, int* __res
             }
         }
     }
-    if (MODE == XBFS_SF) flush_max(&a.st->qmax[(k + 1) % 3], lmax);
+    if (MODE == XBFS_SF && a.track_max) flush_max(&a.st->qmax[(k + 1) % 3], lmax);
 }
 
 template <int MODE>
@@ -500,13 +504,26 @@ __device__ __forceinline__ void ss_count_body(const KArgs& a, int k) {
     unsigned gmax = 0;
     for (long long w = blockIdx.x * (long long)blockDim.x + threadIdx.x; w < a.words;
          w += (long long)gridDim.x * blockDim.x) {
-        const unsigned word = __ldcg(bm + w);
+        unsigned word = __ldcg(bm + w);
         if (!word) continue;
         found += __popc(word);
-        for (unsigned b = word; b; b &= b - 1) {
-            const unsigned d = (unsigned)(__ldg(a.head + w * 32 + __ffs(b) - 1) >> 32);
-            edges += d;
-            gmax = max(gmax, d);
+        // up to 8 head[] loads in flight per step (a dense frontier word holds several bits)
+        while (word) {
+            unsigned long long hv[8];
+#pragma unroll
+            for (int i = 0; i < 8; ++i) {
+                hv[i] = 0ull;
+                if (word) {
+                    hv[i] = __ldg(a.head + w * 32 + __ffs(word) - 1);
+                    word &= word - 1;
+                }
+            }
+#pragma unroll
+            for (int i = 0; i < 8; ++i) {
+                const unsigned d = (unsigned)(hv[i] >> 32);
+                edges += d;
+                gmax = max(gmax, d);
+            }
         }
     }
 #pragma unroll
@@ -518,7 +535,7 @@ __device__ __forceinline__ void ss_count_body(const KArgs& a, int k) {
         atomicAdd(&a.st->acc_found[k % 3], found);
         atomicAdd(&a.st->acc_edges[k % 3], edges);
     }
-    flush_max(&a.st->qmax[(k + 1) % 3], gmax);
+    if (a.track_max) flush_max(&a.st->qmax[(k + 1) % 3], gmax);
 }
 
 __global__ __launch_bounds__(kGenThreads) void k_ss_count(KArgs a) {
@@ -585,7 +602,7 @@ __device__ __forceinline__ void generate_body(const KArgs& a, int k, int role) {
             off += deg;
         }
     }
-    flush_max(&a.st->qmax[role == 0 ? k % 3 : (k + 1) % 3], gmax);
+    if (a.track_max) flush_max(&a.st->qmax[role == 0 ? k % 3 : (k + 1) % 3], gmax);
 }
 
 __global__ __launch_bounds__(kGenThreads) void k_generate(KArgs a, int role) {
@@ -620,7 +637,8 @@ __device__ __forceinline__ void bu_body(const KArgs& a, const int* kp, int* __re
     b.level = level;
     b.parent = parent;
     b.lvl = lvl;
-    bu_chunks<WARPS>(b, sm, [&](long long w, unsigned vis, unsigned f) {
+    b.grab = &a.st->grab[k % 3];
+    bu_chunks<WARPS, true>(b, sm, [&](long long w, unsigned vis, unsigned f) {
         next[w] = f;
         if (f) a.visited[w] = vis | f;
     }, found, edges, probes, fmax);
@@ -637,13 +655,13 @@ __device__ __forceinline__ void bu_body(const KArgs& a, const int* kp, int* __re
         atomicAdd(&a.st->acc_edges[k % 3], edges);
         atomicAdd(&a.st->acc_probes[k % 3], probes);
     }
-    fmax = __reduce_max_sync(FULL, fmax);
-    if (lane == 0 && fmax) {
-        atomic_max_if_greater(&a.st->qmax[(k + 1) % 3], fmax);
+    if (a.track_max) {
+        fmax = __reduce_max_sync(FULL, fmax);
+        if (lane == 0 && fmax) atomic_max_if_greater(&a.st->qmax[(k + 1) % 3], fmax);
     }
 }
 
-__global__ __launch_bounds__(kBuThreads, 5) void k_bu_traverse(KArgs a, int* __restrict__ level,
+__global__ __launch_bounds__(kBuThreads, 4) void k_bu_traverse(KArgs a, int* __restrict__ level,
                                                             int* __restrict__ parent) {
     count_launch(a.st);
     __shared__ BuSmem<kBuThreads / 32> sm;
@@ -847,7 +865,7 @@ __global__ void __cluster_dims__(kSmallCluster, 1, 1) __launch_bounds__(kSmallTh
         st->reached = reached;
         st->arcs_traversed = arcs_tr;
         st->prev_strategy = XBFS_SF;
-        for (int i = 0; i < 3; ++i) st->acc_found[i] = st->acc_edges[i] = st->acc_probes[i] = 0;
+        for (int i = 0; i < 3; ++i) st->acc_found[i] = st->acc_edges[i] = st->acc_probes[i] = st->grab[i] = 0;
         st->fmaxdeg = fmaxdeg;
         st->advanced = st->mirror_host ? 0 : 1;   // graph driver: its k_select node only mirrors
         st->prev_small = 1;
@@ -940,6 +958,7 @@ __global__ __launch_bounds__(kPersistThreads, kPersistBlocks) void k_persist(
             a.st->qctr[(k + 2) % 3] = 0;
             a.st->qmax[(k + 2) % 3] = 0;
             a.st->acc_found[(k + 1) % 3] = a.st->acc_edges[(k + 1) % 3] = a.st->acc_probes[(k + 1) % 3] = 0;
+            a.st->grab[(k + 1) % 3] = 0;
         }
         if (strat != XBFS_BU && !qvalid) {
             generate_body(a, k, 0);
@@ -1224,6 +1243,7 @@ xbfs_status launch_persist(xbfs_graph* g, const KArgs& a, int* level, int* paren
     const unsigned int* noniso = g->nonisolated;
     long long nic = g->nonisolated_count;
     KArgs ka = a;
+    ka.track_max = 0;   // no small-frontier mode inside the persistent kernel
     void* args[] = {&ka, &level, &parent, &noniso, &nic};
     XBFS_CUDA(g, cudaLaunchCooperativeKernel((void*)k_persist, dim3(grid), dim3(kPersistThreads), args,
                                              sizeof(PersistSmem), g->stream));

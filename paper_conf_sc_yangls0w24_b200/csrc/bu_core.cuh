@@ -18,7 +18,16 @@ struct BuView {
     int* level;                       // owned
     int* parent;                      // owned (global ids)
     int lvl;                          // k + 1
+    unsigned long long* grab;         // dynamic chunk counter (zero at level start; DYN instantiation)
 };
+
+#ifndef XBFS_BU_GRAB
+#define XBFS_BU_GRAB 0
+#endif
+// chunks a warp takes per atomic; 0 = static grid-stride, the default: 2/4/8 measured
+// 10-12 % slower at s24 (tools/ab_many.sh: the atomic round trips cost more than the
+// tail imbalance they remove)
+constexpr int kBuGrab = XBFS_BU_GRAB;
 
 // Per-warp shared-memory work lists of one block of WARPS warps (static in the
 // per-level kernels, carved from dynamic shared memory in the persistent one).
@@ -33,7 +42,7 @@ struct BuSmem {
 // publish(w, vis, found_word): store the owned word w of F_{k+1} and update visited.
 // Mutable state (visited, cur) is read through L2 (__ldcg): the persistent
 // driver runs every level inside one kernel, where L1 lines are not refreshed.
-template <int WARPS, class Publish>
+template <int WARPS, bool DYN, class Publish>
 __device__ __forceinline__ void bu_chunks(const BuView& b, BuSmem<WARPS>& sm, Publish publish,
                                           unsigned long long& found, unsigned long long& edges,
                                           unsigned long long& probes, unsigned& fmax) {
@@ -48,12 +57,41 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, BuSmem<WARPS>& sm, Pu
     const long long nchunks = (b.words + kCW - 1) / kCW;
     const long long gw = (blockIdx.x * (long long)blockDim.x + threadIdx.x) >> 5;
     const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
-    for (long long c = gw; c < nchunks; c += nw) {
+    // Chunk order: dynamic (kBuGrab chunks per atomic on b.grab, the next batch
+    // requested one batch ahead, so the level's tail is balanced by work, not by
+    // chunk count) or static grid-stride.
+    const bool dyn = DYN && kBuGrab > 0;
+    unsigned long long nb_l0 = 0;   // lane 0: next batch start, consumed one batch later
+    long long c = gw, bend = 0, cn = 0;
+    if (dyn) {
+        if (lane == 0) c = (long long)atomicAdd(b.grab, (unsigned long long)kBuGrab);
+        c = __shfl_sync(FULL, c, 0);
+        bend = c + kBuGrab;
+        if (lane == 0) nb_l0 = atomicAdd(b.grab, (unsigned long long)kBuGrab);
+    }
+    // the visited words of the warp's next chunk are loaded one iteration ahead
+    // (only this warp writes them), so an empty chunk costs no exposed latency
+    auto load_vis = [&](long long cc) -> unsigned {
+        const long long ww = cc * kCW + lane;
+        return (cc < nchunks && lane < kCW && ww < b.words) ? __ldcg(b.visited + ww) : FULL;
+    };
+    unsigned vis_next = load_vis(c);
+    for (; c < nchunks; c = cn) {
+        if (!dyn) {
+            cn = c + nw;
+        } else if (c + 1 < bend) {
+            cn = c + 1;
+        } else {
+            cn = (long long)__shfl_sync(FULL, nb_l0, 0);
+            bend = cn + kBuGrab;
+            if (lane == 0) nb_l0 = atomicAdd(b.grab, (unsigned long long)kBuGrab);
+        }
         // 1. candidates of kCW bitmap words: ballot/popc compaction into shared memory
         //    (the paper's count + prefix-sum + queue-write "double scan").
         const long long w = c * kCW + lane;
         const bool own = lane < kCW && w < b.words;
-        const unsigned vis = own ? __ldcg(b.visited + w) : FULL;
+        const unsigned vis = vis_next;
+        vis_next = load_vis(cn);
         const unsigned cand = ~vis;
         // fast path: no candidate in the chunk (most chunks in late BU levels); F_{k+1}
         // words start out zero (the stale-bitmap clear of level k-1), so nothing to write

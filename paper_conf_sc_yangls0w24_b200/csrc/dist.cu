@@ -113,7 +113,7 @@ __device__ __forceinline__ int find_parent(const DArgs& a, const unsigned* cur, 
 // ---------------------------------------------------------------- BU
 // The single-GPU bottom-up core (bu_core.cuh) over the owned words; each owned
 // word of F_{k+1} is published to every replica by the lane that owns it.
-__global__ __launch_bounds__(kBuThreads, 5) void k_bu(DArgs a, int k) {
+__global__ __launch_bounds__(kBuThreads, 4) void k_bu(DArgs a, int k) {
     const int slot = (k + 1) % 3;
     unsigned long long found = 0, edges = 0, m = 0, probes = 0;
     unsigned fmax = 0;
@@ -131,8 +131,9 @@ __global__ __launch_bounds__(kBuThreads, 5) void k_bu(DArgs a, int k) {
     b.level = a.level;
     b.parent = a.parent;
     b.lvl = k + 1;
+    b.grab = nullptr;
     __shared__ BuSmem<kBuThreads / 32> sm;
-    bu_chunks<kBuThreads / 32>(b, sm, [&](long long w, unsigned vis, unsigned f) {
+    bu_chunks<kBuThreads / 32, false>(b, sm, [&](long long w, unsigned vis, unsigned f) {
         publish_word(a, slot, w, f);
         if (f) {
             a.vis[w] = vis | f;

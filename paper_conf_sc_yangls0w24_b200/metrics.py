@@ -89,3 +89,32 @@ def bytes_bu(n: int, unvisited: int, probes: int, found: int) -> int:
 def bytes_ss_count(n: int, found: int) -> int:
     """Single-scan count pass: next-frontier bitmap read + 8 B head[] per vertex."""
     return bitmap_bytes(n) + 8 * found
+
+
+def bfs_level_bytes(n: int, strategy, fv, fe, unvisited, probes):
+    """Algorithmic bytes of every level of one BFS given the strategies the
+    selector took (the phases of the persistent kernel): SF and SS
+    read a queue that exists after an SF level (No-Frontier-Generation) and is
+    generated from the frontier bitmap otherwise; SS adds its count pass."""
+    out = []
+    L = len(strategy)
+    for k in range(L):
+        found = fv[k + 1] if k + 1 < L else 0
+        s = strategy[k]
+        queue_valid = k == 0 or strategy[k - 1] == 0
+        b = 0
+        if s != 2 and not queue_valid:
+            b += bytes_generate(n, fv[k], post=False)
+        if s == 0:
+            b += bytes_td_sf(n, fv[k], fe[k], found)
+        elif s == 1:
+            b += bytes_td_ss(n, fv[k], fe[k], found) + bytes_ss_count(n, found)
+        else:
+            b += bytes_bu(n, unvisited[k], probes[k], found)
+        out.append(b)
+    return out
+
+
+def bfs_alg_bytes(n: int, strategy, fv, fe, unvisited, probes) -> int:
+    """Init + every level: the algorithmic bytes of one persistent-kernel launch."""
+    return bytes_init(n) + sum(bfs_level_bytes(n, strategy, fv, fe, unvisited, probes))
