@@ -99,6 +99,11 @@ def load_peaks():
         return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
 
 
+def default_alpha() -> float:
+    from paper_conf_sc_yangls0w24_b200.xbfs import xbfs_run_opts_default
+    return xbfs_run_opts_default().alpha
+
+
 def load_traffic(cfg_name: str, kernel: str):
     """DRAM bytes per launch (dram__bytes_read.sum + dram__bytes_write.sum) of
     `kernel` from the committed `ncu --set full` capture of this bench command
@@ -372,7 +377,7 @@ def run_ours(args):
         "data": "synthetic (seeded Graph500 Kronecker generator, graph seed 1, root seed 2)",
         "config": {"workload": workload_name(args.config), "n_vertices": n, "input_edges": int(src.shape[0]),
                    "arcs": g.arcs, "roots_per_gpu": args.steps, "l2_flush": "512 MiB write before every timed BFS",
-                   "reorder": "degree-desc (P:L153)", "alpha": opts.get("alpha", 0.1),
+                   "reorder": "degree-desc (P:L153)", "alpha": opts.get("alpha", default_alpha()),
                    "bu_stay": opts.get("bu_stay", 1.0),
                    "driver": {0: "persistent (auto)", 1: "host loop", 2: "CUDA-graph loop",
                               3: "persistent"}[args.driver],
@@ -563,7 +568,7 @@ def run_dist(args):
             "data": "synthetic (seeded Graph500 Kronecker generator, graph seed 1, root seed 2)",
             "config": {"workload": workload_name(args.config), "n_vertices": n, "roots": args.steps,
                        "parallelism": f"1D vertex partition x{world} (xbfs_dist, peer-memory frontier exchange)",
-                       "l2_flush": "512 MiB write before every timed BFS", "alpha": opts.get("alpha", 0.1),
+                       "l2_flush": "512 MiB write before every timed BFS", "alpha": opts.get("alpha", default_alpha()),
                        "bu_stay": opts.get("bu_stay", 1.0)},
             "gteps_per_gpu": round(hm / 1e9 / world, 3),
             "gteps_arcs_hmean": round(metrics.harmonic_mean([a / (ms * 1e-3) for (_, ms, _, a, _, _) in per]) / 1e9,

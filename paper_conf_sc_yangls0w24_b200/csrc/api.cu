@@ -71,7 +71,8 @@ int32_t xbfs_compiled_arch(void) {
 void xbfs_run_opts_default(xbfs_run_opts* o) {
     if (!o) return;
     memset(o, 0, sizeof(*o));
-    o->alpha = 0.1;
+    o->alpha = 0.04;      // P:L347 gives 0.1 (MI250X); re-tuned on B200 (reading C-13,
+                          // tools/sweep_selector.py, profiles/r01_selector_sweep.md)
     o->grow = 2.0;        // reading C-10
     o->ratio_min = 1e-3;  // reading C-10
     o->bu_stay = 1.0;     // reading C-11, tuned on B200 (tools/sweep_selector.py); 0 = paper rule

@@ -240,7 +240,7 @@ __device__ __forceinline__ void seed_body(const KArgs& a, int* level, int* paren
     st->fedges = deg;
     st->fprev = 0;
     st->unvisited = nonisolated_count - (deg > 0 ? 1 : 0);
-    for (int i = 0; i < 3; ++i) st->acc_found[i] = st->acc_edges[i] = st->acc_probes[i] = st->grab[i] = 0;
+    for (int i = 0; i < 3; ++i) st->acc_found[i] = st->acc_edges[i] = st->acc_probes[i] = 0;
     st->reached = 0;
     st->arcs_traversed = 0;
     st->nlevels = 0;
@@ -361,7 +361,6 @@ __device__ void select_body(const KArgs& a) {
     st->qctr[(k + 2) % 3] = 0;   // counter of the queue built during level k+1
     st->qmax[(k + 2) % 3] = 0;
     st->acc_found[(k + 1) % 3] = st->acc_edges[(k + 1) % 3] = st->acc_probes[(k + 1) % 3] = 0;
-    st->grab[(k + 1) % 3] = 0;
     sel_store(st, s);
     mirror_host(a, st);
 }
@@ -637,8 +636,7 @@ __device__ __forceinline__ void bu_body(const KArgs& a, const int* kp, int* __re
     b.level = level;
     b.parent = parent;
     b.lvl = lvl;
-    b.grab = &a.st->grab[k % 3];
-    bu_chunks<WARPS, true>(b, sm, [&](long long w, unsigned vis, unsigned f) {
+    bu_chunks<WARPS>(b, sm, [&](long long w, unsigned vis, unsigned f) {
         next[w] = f;
         if (f) a.visited[w] = vis | f;
     }, found, edges, probes, fmax);
@@ -865,7 +863,7 @@ __global__ void __cluster_dims__(kSmallCluster, 1, 1) __launch_bounds__(kSmallTh
         st->reached = reached;
         st->arcs_traversed = arcs_tr;
         st->prev_strategy = XBFS_SF;
-        for (int i = 0; i < 3; ++i) st->acc_found[i] = st->acc_edges[i] = st->acc_probes[i] = st->grab[i] = 0;
+        for (int i = 0; i < 3; ++i) st->acc_found[i] = st->acc_edges[i] = st->acc_probes[i] = 0;
         st->fmaxdeg = fmaxdeg;
         st->advanced = st->mirror_host ? 0 : 1;   // graph driver: its k_select node only mirrors
         st->prev_small = 1;
@@ -958,7 +956,6 @@ __global__ __launch_bounds__(kPersistThreads, kPersistBlocks) void k_persist(
             a.st->qctr[(k + 2) % 3] = 0;
             a.st->qmax[(k + 2) % 3] = 0;
             a.st->acc_found[(k + 1) % 3] = a.st->acc_edges[(k + 1) % 3] = a.st->acc_probes[(k + 1) % 3] = 0;
-            a.st->grab[(k + 1) % 3] = 0;
         }
         if (strat != XBFS_BU && !qvalid) {
             generate_body(a, k, 0);

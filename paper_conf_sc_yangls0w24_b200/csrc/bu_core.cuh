@@ -18,16 +18,8 @@ struct BuView {
     int* level;                       // owned
     int* parent;                      // owned (global ids)
     int lvl;                          // k + 1
-    unsigned long long* grab;         // dynamic chunk counter (zero at level start; DYN instantiation)
 };
 
-#ifndef XBFS_BU_GRAB
-#define XBFS_BU_GRAB 0
-#endif
-// chunks a warp takes per atomic; 0 = static grid-stride, the default: 2/4/8 measured
-// 10-12 % slower at s24 (tools/ab_many.sh: the atomic round trips cost more than the
-// tail imbalance they remove)
-constexpr int kBuGrab = XBFS_BU_GRAB;
 
 // Per-warp shared-memory work lists of one block of WARPS warps (static in the
 // per-level kernels, carved from dynamic shared memory in the persistent one).
@@ -42,7 +34,7 @@ struct BuSmem {
 // publish(w, vis, found_word): store the owned word w of F_{k+1} and update visited.
 // Mutable state (visited, cur) is read through L2 (__ldcg): the persistent
 // driver runs every level inside one kernel, where L1 lines are not refreshed.
-template <int WARPS, bool DYN, class Publish>
+template <int WARPS, class Publish>
 __device__ __forceinline__ void bu_chunks(const BuView& b, BuSmem<WARPS>& sm, Publish publish,
                                           unsigned long long& found, unsigned long long& edges,
                                           unsigned long long& probes, unsigned& fmax) {
@@ -57,202 +49,192 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, BuSmem<WARPS>& sm, Pu
     const long long nchunks = (b.words + kCW - 1) / kCW;
     const long long gw = (blockIdx.x * (long long)blockDim.x + threadIdx.x) >> 5;
     const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
-    // Chunk order: dynamic (kBuGrab chunks per atomic on b.grab, the next batch
-    // requested one batch ahead, so the level's tail is balanced by work, not by
-    // chunk count) or static grid-stride.
-    const bool dyn = DYN && kBuGrab > 0;
-    unsigned long long nb_l0 = 0;   // lane 0: next batch start, consumed one batch later
-    long long c = gw, bend = 0, cn = 0;
-    if (dyn) {
-        if (lane == 0) c = (long long)atomicAdd(b.grab, (unsigned long long)kBuGrab);
-        c = __shfl_sync(FULL, c, 0);
-        bend = c + kBuGrab;
-        if (lane == 0) nb_l0 = atomicAdd(b.grab, (unsigned long long)kBuGrab);
-    }
-    // the visited words of the warp's next chunk are loaded one iteration ahead
-    // (only this warp writes them), so an empty chunk costs no exposed latency
-    auto load_vis = [&](long long cc) -> unsigned {
-        const long long ww = cc * kCW + lane;
-        return (cc < nchunks && lane < kCW && ww < b.words) ? __ldcg(b.visited + ww) : FULL;
+    // Static chunk order: warp gw takes chunks gw, gw + nw, ... in groups of 4
+    // (32 lanes = 4 chunks x kCW words): one load round trip tells which of the 4
+    // chunks hold candidates, and the next group's words are loaded one group
+    // ahead (only this warp writes them), so chunks without candidates (most of
+    // them in late BU levels) cost no exposed latency.
+    static_assert(kCW == 8, "4 chunks of 8 words per warp load");
+    auto load_group = [&](long long g0) -> unsigned {
+        const long long cc = g0 + (long long)(lane >> 3) * nw;
+        const long long ww = cc * kCW + (lane & 7);
+        return (cc < nchunks && ww < b.words) ? __ldcg(b.visited + ww) : FULL;
     };
-    unsigned vis_next = load_vis(c);
-    for (; c < nchunks; c = cn) {
-        if (!dyn) {
-            cn = c + nw;
-        } else if (c + 1 < bend) {
-            cn = c + 1;
-        } else {
-            cn = (long long)__shfl_sync(FULL, nb_l0, 0);
-            bend = cn + kBuGrab;
-            if (lane == 0) nb_l0 = atomicAdd(b.grab, (unsigned long long)kBuGrab);
-        }
-        // 1. candidates of kCW bitmap words: ballot/popc compaction into shared memory
-        //    (the paper's count + prefix-sum + queue-write "double scan").
-        const long long w = c * kCW + lane;
-        const bool own = lane < kCW && w < b.words;
-        const unsigned vis = vis_next;
-        vis_next = load_vis(cn);
-        const unsigned cand = ~vis;
-        // fast path: no candidate in the chunk (most chunks in late BU levels); F_{k+1}
-        // words start out zero (the stale-bitmap clear of level k-1), so nothing to write
-        if (__ballot_sync(FULL, cand != 0u) == 0u) continue;
-        const int cnt = __popc(cand);
-        int incl = cnt;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            const int t = __shfl_up_sync(FULL, incl, o);
-            if (lane >= o) incl += t;
-        }
-        const int total = __shfl_sync(FULL, incl, 31);
-        int pos = incl - cnt;
-        for (unsigned bits = cand; bits; bits &= bits - 1) s_list[wib][pos++] = (int)(w * 32 + __ffs(bits) - 1);
-        if (lane < kCW) s_found[wib][lane] = 0;
-        __syncwarp();
-        // 2. first probe of every candidate, kBuFirstIlp candidates per lane in flight:
-        //    head[v] (deg << 32 | first stored neighbour) is a dense array read in
-        //    candidate order, so a hit (the common case after the degree-desc
-        //    re-arrangement) never touches row_ptr or col.  Misses with more
-        //    arcs are compacted in place at the front of s_list.
-        int nmiss = 0;
-        for (int base = 0; base < total; base += 32 * kBuFirstIlp) {
-            int vv[kBuFirstIlp];
-            unsigned long long hv[kBuFirstIlp];
-            unsigned wd[kBuFirstIlp];
-#pragma unroll
-            for (int g = 0; g < kBuFirstIlp; ++g) {
-                const int idx = base + g * 32 + lane;
-                vv[g] = idx < total ? s_list[wib][idx] : -1;
+    unsigned grp_next = load_group(gw);
+    for (long long g0 = gw; g0 < nchunks; g0 += 4 * nw) {
+        const unsigned grp = grp_next;
+        grp_next = load_group(g0 + 4 * nw);
+        unsigned has = __ballot_sync(FULL, grp != FULL);   // lanes whose word has a candidate
+        for (int j = 0; has; ++j, has >>= 8) {
+            if ((has & 0xffu) == 0u) continue;
+            const long long c = g0 + (long long)j * nw;
+            const unsigned vis_j = __shfl_sync(FULL, grp, (j << 3) | (lane & 7));
+            // 1. candidates of kCW bitmap words: ballot/popc compaction into shared memory
+            //    (the paper's count + prefix-sum + queue-write "double scan").
+            const long long w = c * kCW + lane;
+            const bool own = lane < kCW && w < b.words;
+            const unsigned vis = own ? vis_j : FULL;
+            const unsigned cand = ~vis;
+            // (chunks without a candidate were skipped above: F_{k+1} words start out
+            // zero, the stale-bitmap clear of level k-1, so there is nothing to write)
+            const int cnt = __popc(cand);
+            int incl = cnt;
+    #pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const int t = __shfl_up_sync(FULL, incl, o);
+                if (lane >= o) incl += t;
             }
-#pragma unroll
-            for (int g = 0; g < kBuFirstIlp; ++g) hv[g] = vv[g] >= 0 ? __ldg(b.head + vv[g]) : 0ull;
-#pragma unroll
-            for (int g = 0; g < kBuFirstIlp; ++g) {
-                const int fu = (int)(unsigned)hv[g];
-                wd[g] = vv[g] >= 0 ? __ldcg(b.cur + (fu >> 5)) : 0u;
-            }
-            __syncwarp();   // every read of this round is done before the in-place compaction
-#pragma unroll
-            for (int g = 0; g < kBuFirstIlp; ++g) {
-                const int v = vv[g];
-                bool miss = false;
-                if (v >= 0) {
+            const int total = __shfl_sync(FULL, incl, 31);
+            int pos = incl - cnt;
+            for (unsigned bits = cand; bits; bits &= bits - 1) s_list[wib][pos++] = (int)(w * 32 + __ffs(bits) - 1);
+            if (lane < kCW) s_found[wib][lane] = 0;
+            __syncwarp();
+            // 2. first probe of every candidate, kBuFirstIlp candidates per lane in flight:
+            //    head[v] (deg << 32 | first stored neighbour) is a dense array read in
+            //    candidate order, so a hit (the common case after the degree-desc
+            //    re-arrangement) never touches row_ptr or col.  Misses with more
+            //    arcs are compacted in place at the front of s_list.
+            int nmiss = 0;
+            for (int base = 0; base < total; base += 32 * kBuFirstIlp) {
+                int vv[kBuFirstIlp];
+                unsigned long long hv[kBuFirstIlp];
+                unsigned wd[kBuFirstIlp];
+    #pragma unroll
+                for (int g = 0; g < kBuFirstIlp; ++g) {
+                    const int idx = base + g * 32 + lane;
+                    vv[g] = idx < total ? s_list[wib][idx] : -1;
+                }
+    #pragma unroll
+                for (int g = 0; g < kBuFirstIlp; ++g) hv[g] = vv[g] >= 0 ? __ldg(b.head + vv[g]) : 0ull;
+    #pragma unroll
+                for (int g = 0; g < kBuFirstIlp; ++g) {
                     const int fu = (int)(unsigned)hv[g];
-                    const long long d = (long long)(hv[g] >> 32);
-                    if ((wd[g] >> (fu & 31)) & 1u) {
+                    wd[g] = vv[g] >= 0 ? __ldcg(b.cur + (fu >> 5)) : 0u;
+                }
+                __syncwarp();   // every read of this round is done before the in-place compaction
+    #pragma unroll
+                for (int g = 0; g < kBuFirstIlp; ++g) {
+                    const int v = vv[g];
+                    bool miss = false;
+                    if (v >= 0) {
+                        const int fu = (int)(unsigned)hv[g];
+                        const long long d = (long long)(hv[g] >> 32);
+                        if ((wd[g] >> (fu & 31)) & 1u) {
+                            b.level[v] = b.lvl;
+                            b.parent[v] = fu;
+                            atomicOr(&s_found[wib][(v >> 5) - c * kCW], 1u << (v & 31));
+                            edges += (unsigned long long)d;
+                            fmax = max(fmax, (unsigned)d);
+                            ++found;
+                            probes += 1;
+                        } else if (d == 1) {
+                            probes += 1;
+                        } else {
+                            miss = true;
+                        }
+                    }
+                    const unsigned mm = __ballot_sync(FULL, miss);
+                    if (miss) s_list[wib][nmiss + __popc(mm & lt)] = v;
+                    nmiss += __popc(mm);
+                }
+            }
+            __syncwarp();
+            // 3. the misses: lane-per-candidate, kBuBatch arcs per step in stored
+            //    order from the second arc on; a lane that finishes takes the next
+            //    candidate, so lanes stay busy.
+            int v = -1, nxt = 0, nhard = 0;
+            long long rs = 0, re = 0, p = 0;
+            for (;;) {
+                const unsigned need = __ballot_sync(FULL, v < 0);
+                if (v < 0) {
+                    const int idx = nxt + __popc(need & lt);
+                    if (idx < nmiss) {
+                        v = s_list[wib][idx];
+                        rs = b.row_ptr[v];
+                        re = b.row_ptr[v + 1];
+                        p = rs + 1;
+                    }
+                }
+                nxt += __popc(need);
+                if (!__any_sync(FULL, v >= 0)) break;
+                bool to_hard = false;
+                if (v >= 0) {
+                    const long long end = min(re, p + kBuBatch);
+                    int u[kBuBatch];
+                    unsigned wd[kBuBatch];
+    #pragma unroll
+                    for (int j = 0; j < kBuBatch; ++j) u[j] = (p + j < end) ? __ldg(b.col + p + j) : -1;
+    #pragma unroll
+                    for (int j = 0; j < kBuBatch; ++j) wd[j] = u[j] >= 0 ? __ldcg(b.cur + (u[j] >> 5)) : 0u;
+                    int hit = -1;
+    #pragma unroll
+                    for (int j = kBuBatch - 1; j >= 0; --j)
+                        if (u[j] >= 0 && ((wd[j] >> (u[j] & 31)) & 1u)) hit = j;   // first hit in row order
+                    if (hit >= 0) {
+                        int pu = u[0];
+    #pragma unroll
+                        for (int j = 1; j < kBuBatch; ++j) if (j == hit) pu = u[j];
                         b.level[v] = b.lvl;
-                        b.parent[v] = fu;
+                        b.parent[v] = pu;
                         atomicOr(&s_found[wib][(v >> 5) - c * kCW], 1u << (v & 31));
-                        edges += (unsigned long long)d;
-                        fmax = max(fmax, (unsigned)d);
+                        edges += (unsigned long long)(re - rs);
+                        fmax = max(fmax, (unsigned)(re - rs));
                         ++found;
-                        probes += 1;
-                    } else if (d == 1) {
-                        probes += 1;
+                        probes += (unsigned long long)(p + hit + 1 - rs);
+                        v = -1;
+                    } else if (end == re) {
+                        probes += (unsigned long long)(re - rs);
+                        v = -1;
+                    } else if (re - end > kBuHardMin) {
+                        to_hard = true;
                     } else {
-                        miss = true;
+                        p = end;
                     }
                 }
-                const unsigned mm = __ballot_sync(FULL, miss);
-                if (miss) s_list[wib][nmiss + __popc(mm & lt)] = v;
-                nmiss += __popc(mm);
-            }
-        }
-        __syncwarp();
-        // 3. the misses: lane-per-candidate, kBuBatch arcs per step in stored
-        //    order from the second arc on; a lane that finishes takes the next
-        //    candidate, so lanes stay busy.
-        int v = -1, nxt = 0, nhard = 0;
-        long long rs = 0, re = 0, p = 0;
-        for (;;) {
-            const unsigned need = __ballot_sync(FULL, v < 0);
-            if (v < 0) {
-                const int idx = nxt + __popc(need & lt);
-                if (idx < nmiss) {
-                    v = s_list[wib][idx];
-                    rs = b.row_ptr[v];
-                    re = b.row_ptr[v + 1];
-                    p = rs + 1;
-                }
-            }
-            nxt += __popc(need);
-            if (!__any_sync(FULL, v >= 0)) break;
-            bool to_hard = false;
-            if (v >= 0) {
-                const long long end = min(re, p + kBuBatch);
-                int u[kBuBatch];
-                unsigned wd[kBuBatch];
-#pragma unroll
-                for (int j = 0; j < kBuBatch; ++j) u[j] = (p + j < end) ? __ldg(b.col + p + j) : -1;
-#pragma unroll
-                for (int j = 0; j < kBuBatch; ++j) wd[j] = u[j] >= 0 ? __ldcg(b.cur + (u[j] >> 5)) : 0u;
-                int hit = -1;
-#pragma unroll
-                for (int j = kBuBatch - 1; j >= 0; --j)
-                    if (u[j] >= 0 && ((wd[j] >> (u[j] & 31)) & 1u)) hit = j;   // first hit in row order
-                if (hit >= 0) {
-                    int pu = u[0];
-#pragma unroll
-                    for (int j = 1; j < kBuBatch; ++j) if (j == hit) pu = u[j];
-                    b.level[v] = b.lvl;
-                    b.parent[v] = pu;
-                    atomicOr(&s_found[wib][(v >> 5) - c * kCW], 1u << (v & 31));
-                    edges += (unsigned long long)(re - rs);
-                    fmax = max(fmax, (unsigned)(re - rs));
-                    ++found;
-                    probes += (unsigned long long)(p + hit + 1 - rs);
+                const unsigned hm = __ballot_sync(FULL, to_hard);
+                if (to_hard) {
+                    const int hi = nhard + __popc(hm & lt);
+                    s_hard[wib][hi] = v;
+                    s_hoff[wib][hi] = (int)(p + kBuBatch - rs);
                     v = -1;
-                } else if (end == re) {
-                    probes += (unsigned long long)(re - rs);
-                    v = -1;
-                } else if (re - end > kBuHardMin) {
-                    to_hard = true;
-                } else {
-                    p = end;
                 }
+                nhard += __popc(hm);
             }
-            const unsigned hm = __ballot_sync(FULL, to_hard);
-            if (to_hard) {
-                const int hi = nhard + __popc(hm & lt);
-                s_hard[wib][hi] = v;
-                s_hoff[wib][hi] = (int)(p + kBuBatch - rs);
-                v = -1;
-            }
-            nhard += __popc(hm);
-        }
-        __syncwarp();
-        // 4. long unresolved rows: the whole warp probes 32 arcs per step, first hit wins
-        for (int h = 0; h < nhard; ++h) {
-            const int hv = s_hard[wib][h];
-            const long long hrs = b.row_ptr[hv], hre = b.row_ptr[hv + 1];
-            bool hit_any = false;
-            for (long long base = hrs + s_hoff[wib][h]; base < hre; base += 32) {
-                const long long pp = base + lane;
-                const int u = pp < hre ? __ldg(b.col + pp) : -1;
-                const bool hit = u >= 0 && ((__ldcg(b.cur + (u >> 5)) >> (u & 31)) & 1u);
-                const unsigned m = __ballot_sync(FULL, hit);
-                if (m) {
-                    const int first = __ffs(m) - 1;
-                    if (lane == first) {
-                        b.level[hv] = b.lvl;
-                        b.parent[hv] = u;
-                        atomicOr(&s_found[wib][(hv >> 5) - c * kCW], 1u << (hv & 31));
-                        edges += (unsigned long long)(hre - hrs);
-                        fmax = max(fmax, (unsigned)(hre - hrs));
-                        ++found;
-                        probes += (unsigned long long)(pp + 1 - hrs);
+            __syncwarp();
+            // 4. long unresolved rows: the whole warp probes 32 arcs per step, first hit wins
+            for (int h = 0; h < nhard; ++h) {
+                const int hv = s_hard[wib][h];
+                const long long hrs = b.row_ptr[hv], hre = b.row_ptr[hv + 1];
+                bool hit_any = false;
+                for (long long base = hrs + s_hoff[wib][h]; base < hre; base += 32) {
+                    const long long pp = base + lane;
+                    const int u = pp < hre ? __ldg(b.col + pp) : -1;
+                    const bool hit = u >= 0 && ((__ldcg(b.cur + (u >> 5)) >> (u & 31)) & 1u);
+                    const unsigned m = __ballot_sync(FULL, hit);
+                    if (m) {
+                        const int first = __ffs(m) - 1;
+                        if (lane == first) {
+                            b.level[hv] = b.lvl;
+                            b.parent[hv] = u;
+                            atomicOr(&s_found[wib][(hv >> 5) - c * kCW], 1u << (hv & 31));
+                            edges += (unsigned long long)(hre - hrs);
+                            fmax = max(fmax, (unsigned)(hre - hrs));
+                            ++found;
+                            probes += (unsigned long long)(pp + 1 - hrs);
+                        }
+                        hit_any = true;
+                        break;
                     }
-                    hit_any = true;
-                    break;
                 }
+                if (!hit_any && lane == 0) probes += (unsigned long long)(hre - hrs);
             }
-            if (!hit_any && lane == 0) probes += (unsigned long long)(hre - hrs);
+            __syncwarp();
+            if (own) {
+                const unsigned f = s_found[wib][lane];
+                if (f) publish(w, vis, f);   // zero words are already zero in every replica
+            }
+            __syncwarp();
         }
-        __syncwarp();
-        if (own) {
-            const unsigned f = s_found[wib][lane];
-            if (f) publish(w, vis, f);   // zero words are already zero in every replica
-        }
-        __syncwarp();
     }
 }
 

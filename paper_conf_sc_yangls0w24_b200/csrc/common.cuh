@@ -69,7 +69,6 @@ struct DevState {
     long long unvisited;         // U_k (non-isolated, unvisited)
     unsigned long long acc_found[3], acc_edges[3], acc_probes[3];  // BU / SS-count accumulators:
                                  // level k adds into slot k%3; slot (k+1)%3 is zeroed before level k+1
-    unsigned long long grab[3];  // BU dynamic chunk counter of level k (slot k%3, zeroed like acc)
     long long reached, arcs_traversed;
     unsigned int launches;       // library kernels launched (device-counted)
     int nlevels;

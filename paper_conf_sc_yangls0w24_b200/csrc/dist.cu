@@ -131,9 +131,8 @@ __global__ __launch_bounds__(kBuThreads, 4) void k_bu(DArgs a, int k) {
     b.level = a.level;
     b.parent = a.parent;
     b.lvl = k + 1;
-    b.grab = nullptr;
     __shared__ BuSmem<kBuThreads / 32> sm;
-    bu_chunks<kBuThreads / 32, false>(b, sm, [&](long long w, unsigned vis, unsigned f) {
+    bu_chunks<kBuThreads / 32>(b, sm, [&](long long w, unsigned vis, unsigned f) {
         publish_word(a, slot, w, f);
         if (f) {
             a.vis[w] = vis | f;

@@ -40,7 +40,7 @@ def test_compiled_for_sm100a(xb):
 
 def test_defaults(xb):
     o = xb.xbfs_run_opts_default()
-    assert o.alpha == 0.1 and o.force_strategy == -1   # alpha from P:L347
+    assert o.alpha == 0.04 and o.force_strategy == -1   # P:L347 uses 0.1; B200-tuned (reading C-13)
 
 
 def test_invalid_arguments_do_not_touch_cuda(xb):

@@ -26,8 +26,10 @@ def line_map(so: str, func: str):
         start = full.find(f".text.{func}:")
         if start < 0:
             continue
-        end = full.find("\n.section", start + 1)
-        out = full[start: end if end > 0 else len(full)]
+        lines = full[start:].splitlines()
+        stop = next((i for i, l in enumerate(lines[1:], 1)
+                     if l.startswith(".text.") or l.lstrip().startswith(".section")), len(lines))
+        out = "\n".join(lines[:stop])
         m, cur = {}, None
         for ln in out.splitlines():
             a = re.match(r'\s*//## File "([^"]+)", line (\d+)', ln)
