@@ -40,8 +40,10 @@ def _check_run(g, og, src, dst, root, **opts):
     # counters against the oracle's per-level facts
     fs, fe = oracle.level_stats(og, ref)
     assert st.num_levels == nl
-    assert st.frontier_vertices == fs.tolist()
-    assert st.frontier_edges == fe.tolist()
+    cap = len(st.frontier_vertices)          # per-level log: the first min(nl, capacity) levels
+    assert cap == min(nl, 1 << 14)
+    assert st.frontier_vertices == fs.tolist()[:cap]
+    assert st.frontier_edges == fe.tolist()[:cap]
     assert st.vertices_reached == int((ref >= 0).sum())
     assert st.arcs_traversed == int(fe.sum())
     assert st.input_edges_traversed == oracle.input_edges(src, ref)
@@ -272,4 +274,40 @@ def test_persistent_driver_level_times(xb):
         assert sum(st.level_ms) <= st.elapsed_ms * 1.01
         st = _check_run(g, og, src, dst, root, driver=1)
         assert st.kernel_launches > 1 and all(t == 0 for t in st.level_ms)
+    g.close()
+
+
+def test_deep_levels_escape_the_level_store(xb):
+    """A path deeper than the 2-byte level store (kLvMax = 32765 levels): the
+    deep levels go straight to level[] / parent[] and the epilogue keeps them;
+    BU parents below and above the limit are found from mixed entries."""
+    n = 32_800
+    src = np.arange(n - 1, dtype=np.uint32)
+    dst = src + 1
+    og = oracle.build_csr(n, src, dst)
+    g = xb.Graph(_dev(src), _dev(dst), n)
+    for root, opts in ((0, dict()), (0, dict(force_strategy=2)), (n - 1, dict(force_strategy=1)),
+                       (0, dict(driver=1, small_edges=0)), (n // 2, dict())):
+        st = _check_run(g, og, src, dst, root, **opts)
+        assert st.num_levels == max(root, n - 1 - root) + 1
+    g.close()
+
+
+def test_unaligned_output_arrays(xb):
+    """The epilogue writes 16-byte groups only when both outputs are 16-byte
+    aligned; offset views take the scalar path and still get every element."""
+    src, dst, n = synth.kronecker(11, seed=9)
+    n += 3                                   # N not a multiple of 4; 3 isolated vertices
+    og = oracle.build_csr(n, src, dst)
+    g = xb.Graph(_dev(src), _dev(dst), n)
+    lbuf = torch.full((n + 1,), 7, dtype=torch.int32, device="cuda")
+    pbuf = torch.full((n + 1,), 7, dtype=torch.int32, device="cuda")
+    for root in synth.roots(n - 3, src, dst, 3, root_seed=1):
+        for opts in (dict(), dict(driver=1), dict(force_strategy=2)):
+            level, parent, _ = g.run(int(root), lbuf[1:], pbuf[1:], stats=True, **opts)
+            lv, pa = level.cpu().numpy(), parent.cpu().numpy()
+            ref, _, _ = oracle.bfs(og, int(root))
+            assert np.array_equal(lv, ref)
+            assert oracle.validate(og, src, dst, int(root), lv, pa) == 0
+            assert int(lbuf[0]) == 7 and int(pbuf[0]) == 7
     g.close()
