@@ -75,6 +75,12 @@ typedef struct {
     int32_t plan_len;        /* > 0: strategy plan for levels [0, plan_len) (host-loop driver only) */
     const int8_t* plan;      /* host array: plan[k] in {-1 selector, 0 SF, 1 SS, 2 BU} overrides the
                                 strategy of level k (forced-strategy studies, Tab VI) */
+    int32_t lookahead;       /* 1: bottom-up look-ahead ("proactive") update, SURVEY f1:
+                                a BU step also sets to level k+2 every candidate whose whole row has
+                                no F_k vertex but a vertex this same pass already put in F_{k+1}.
+                                Levels stay exact; parents of those vertices are that neighbour.
+                                Persistent driver only (driver 0 / 3, no plan, no per-launch
+                                profiling): XBFS_ERR_INVALID_ARG otherwise.  Default 0. */
 } xbfs_run_opts;
 
 /* Per-run statistics; filled when a non-NULL pointer is passed (xbfs_run then
@@ -104,6 +110,8 @@ typedef struct {
     /* [level_capacity] device time of level k in ms (persistent driver: %globaltimer
      * stamps at the grid barrier ending each level; 0 under the other drivers) */
     float* level_ms;
+    /* [level_capacity] vertices step k set to level k+2 through the BU look-ahead (0 if off) */
+    int64_t* lookahead_found;
 } xbfs_run_stats;
 
 /* kernel ids reported in xbfs_run_stats.kernel_id */

@@ -39,6 +39,7 @@ xbfs::KArgs xbfs_graph::kargs() const {
     a.visited = visited;
     const long long stride = (words + 31) / 32 * 32;  // 128-byte aligned bitmaps (uint4 access)
     for (int i = 0; i < 3; ++i) a.fb[i] = fb + i * stride;
+    a.la = fb + 3 * stride;
     for (int i = 0; i < 3; ++i) {
         a.qv[i] = qv + i * n;
         a.qoff[i] = qoff + i * n;

@@ -26,6 +26,7 @@
 #include <cooperative_groups.h>
 
 #include <algorithm>
+#include <type_traits>
 
 #include "common.cuh"
 #include "bu_core.cuh"
@@ -187,6 +188,7 @@ __device__ __forceinline__ void init_body(const KArgs& a, int* __restrict__ leve
         a.fb[0][w] = 0;
         a.fb[1][w] = 0;
         a.fb[2][w] = 0;
+        a.la[w] = 0;
     }
 }
 
@@ -240,7 +242,10 @@ __device__ __forceinline__ void seed_body(const KArgs& a, int* level, int* paren
     st->fedges = deg;
     st->fprev = 0;
     st->unvisited = nonisolated_count - (deg > 0 ? 1 : 0);
-    for (int i = 0; i < 3; ++i) st->acc_found[i] = st->acc_edges[i] = st->acc_probes[i] = 0;
+    for (int i = 0; i < 3; ++i) {
+        st->acc_found[i] = st->acc_edges[i] = st->acc_probes[i] = 0;
+        st->acc_la_found[i] = st->acc_la_edges[i] = 0;
+    }
     st->reached = 0;
     st->arcs_traversed = 0;
     st->nlevels = 0;
@@ -259,8 +264,9 @@ __global__ void k_seed(KArgs a, int* level, int* parent, long long nonisolated_c
 // The level state the selector evolves (one copy per CTA in the persistent
 // driver, where every CTA computes the same decision from the same counters).
 struct SelState {
-    int k, strategy, queue_valid, done, prev_strategy, nlevels, prev_small, pad_;
+    int k, strategy, queue_valid, done, prev_strategy, nlevels, prev_small, prefill;
     long long fsize, fedges, fprev, unvisited, reached, arcs_traversed;
+    long long la_cf, la_ce;    // look-ahead vertices (count, degree sum) merged into F_{k+1} before level k
     unsigned fmaxdeg;
 };
 
@@ -283,12 +289,27 @@ __device__ __forceinline__ void select_step(const KArgs& a, SelState& s, bool lo
         ne = (long long)(q & ((1ull << a.dbits) - 1ull));
         s.queue_valid = 1;
     }
+    // look-ahead (persistent driver): vertices of F_{k+1} that BU step k-1 already
+    // set (level k+1) were merged into the F_{k+1} bitmap before this level; the
+    // count pass of SS saw them, the BU / SF counters did not, and an SF queue
+    // lacks them.
+    const long long carry_f = s.la_cf;
+    if (carry_f) {
+        if (strat != XBFS_SS) { nf += carry_f; ne += s.la_ce; }
+        s.queue_valid = 0;
+    }
+    long long laf = 0, lae = 0;
+    if (strat == XBFS_BU && st->lookahead) {
+        laf = (long long)__ldcg(&st->acc_la_found[k % 3]);
+        lae = (long long)__ldcg(&st->acc_la_edges[k % 3]);
+    }
     if (log_it && k < kLogCap) {
         LevelRec r;
         r.fsize = s.fsize;
         r.fedges = s.fedges;
         r.unvisited = s.unvisited;
         r.probes = strat == XBFS_BU ? (long long)__ldcg(&st->acc_probes[k % 3]) : 0;
+        r.la_found = laf;
         r.strategy = strat;
         r.pad = 0;
         r.t_ns = t_ns;
@@ -302,7 +323,10 @@ __device__ __forceinline__ void select_step(const KArgs& a, SelState& s, bool lo
     s.fprev = s.fsize;
     s.fsize = nf;
     s.fedges = ne;
-    s.unvisited -= nf;
+    s.unvisited -= nf - carry_f + laf;   // newly visited during level k
+    s.la_cf = laf;
+    s.la_ce = lae;
+    s.prefill = laf > 0;
     s.prev_strategy = strat;
     s.k = k + 1;
     s.fmaxdeg = __ldcg(&st->qmax[(k + 1) % 3]);
@@ -329,6 +353,8 @@ __device__ __forceinline__ void sel_load(const DevState* st, SelState& s) {
     s.reached = __ldcg(&st->reached);
     s.arcs_traversed = __ldcg(&st->arcs_traversed);
     s.fmaxdeg = __ldcg(&st->fmaxdeg);
+    s.prefill = 0;
+    s.la_cf = s.la_ce = 0;   // look-ahead runs only in the persistent driver, whose state never leaves the kernel
 }
 
 __device__ __forceinline__ void sel_store(DevState* st, const SelState& s) {
@@ -361,6 +387,7 @@ __device__ void select_body(const KArgs& a) {
     st->qctr[(k + 2) % 3] = 0;   // counter of the queue built during level k+1
     st->qmax[(k + 2) % 3] = 0;
     st->acc_found[(k + 1) % 3] = st->acc_edges[(k + 1) % 3] = st->acc_probes[(k + 1) % 3] = 0;
+    st->acc_la_found[(k + 1) % 3] = st->acc_la_edges[(k + 1) % 3] = 0;
     sel_store(st, s);
     mirror_host(a, st);
 }
@@ -616,9 +643,9 @@ __global__ __launch_bounds__(kGenThreads) void k_generate(KArgs a, int role) {
 // kp: where k lives (DevState or the persistent CTA's selector copy); it is
 // re-read for the epilogue instead of keeping k live across the traversal
 // (one register less: the per-level kernel runs at 48 without spills).
-template <int WARPS>
+template <int WARPS, bool LA, class Smem>
 __device__ __forceinline__ void bu_body(const KArgs& a, const int* kp, int* __restrict__ level,
-                                        int* __restrict__ parent, BuSmem<WARPS>& sm) {
+                                        int* __restrict__ parent, Smem& sm, bool prefill) {
     int k = *(const volatile int*)kp;
     clear_stale(a, k);
     const unsigned int* __restrict__ cur = a.fb[k % 3];
@@ -626,8 +653,10 @@ __device__ __forceinline__ void bu_body(const KArgs& a, const int* kp, int* __re
     const int lvl = k + 1;
     unsigned long long found = 0, edges = 0, probes = 0;
     unsigned fmax = 0;
+    BuLa la;
     BuView b;
     b.cur = cur;
+    b.nxt = next;
     b.visited = a.visited;
     b.words = a.words;
     b.head = a.head;
@@ -636,16 +665,24 @@ __device__ __forceinline__ void bu_body(const KArgs& a, const int* kp, int* __re
     b.level = level;
     b.parent = parent;
     b.lvl = lvl;
-    bu_chunks<WARPS>(b, sm, [&](long long w, unsigned vis, unsigned f) {
-        next[w] = f;
-        if (f) a.visited[w] = vis | f;
-    }, found, edges, probes, fmax);
+    // prefill: F_{k+1} already holds look-ahead vertices of step k-1 (OR into it)
+    const bool pf = LA && prefill;
+    bu_chunks<WARPS, LA>(b, sm, [&](long long w, unsigned vis, unsigned f, unsigned lf) {
+        if (pf) f |= __ldcg(next + w);
+        if (f) next[w] = f;
+        a.visited[w] = vis | f | lf;
+        if (LA && lf) a.la[w] = lf;
+    }, found, edges, probes, fmax, la);
     const int lane = threadIdx.x & 31;
 #pragma unroll
     for (int o = 16; o; o >>= 1) {
         found += __shfl_xor_sync(FULL, found, o);
         edges += __shfl_xor_sync(FULL, edges, o);
         probes += __shfl_xor_sync(FULL, probes, o);
+        if (LA) {
+            la.found += __shfl_xor_sync(FULL, la.found, o);
+            la.edges += __shfl_xor_sync(FULL, la.edges, o);
+        }
     }
     k = *(const volatile int*)kp;
     if (lane == 0 && (found | edges | probes)) {
@@ -653,9 +690,28 @@ __device__ __forceinline__ void bu_body(const KArgs& a, const int* kp, int* __re
         atomicAdd(&a.st->acc_edges[k % 3], edges);
         atomicAdd(&a.st->acc_probes[k % 3], probes);
     }
+    if (LA && lane == 0 && la.found) {
+        atomicAdd(&a.st->acc_la_found[k % 3], la.found);
+        atomicAdd(&a.st->acc_la_edges[k % 3], la.edges);
+    }
     if (a.track_max) {
         fmax = __reduce_max_sync(FULL, fmax);
         if (lane == 0 && fmax) atomic_max_if_greater(&a.st->qmax[(k + 1) % 3], fmax);
+    }
+}
+
+// Look-ahead merge (persistent driver, after a BU step with look-ahead
+// discoveries): F_{k+2} |= la, la = 0.  F_{k+2}'s bitmap was cleared during step
+// k (the stale-map clear); the grid barrier that follows orders it before step k+1.
+__device__ __forceinline__ void la_merge(const KArgs& a, int knext) {
+    unsigned int* f2 = a.fb[(knext + 1) % 3];
+    for (long long w = blockIdx.x * (long long)blockDim.x + threadIdx.x; w < a.words;
+         w += (long long)gridDim.x * blockDim.x) {
+        const unsigned x = __ldcg(a.la + w);
+        if (x) {
+            f2[w] = __ldcg(f2 + w) | x;
+            a.la[w] = 0;
+        }
     }
 }
 
@@ -663,7 +719,7 @@ __global__ __launch_bounds__(kBuThreads, 4) void k_bu_traverse(KArgs a, int* __r
                                                             int* __restrict__ parent) {
     count_launch(a.st);
     __shared__ BuSmem<kBuThreads / 32> sm;
-    bu_body<kBuThreads / 32>(a, &a.st->k, level, parent, sm);
+    bu_body<kBuThreads / 32, false>(a, &a.st->k, level, parent, sm, false);
 }
 
 // ---------------------------------------------------------------- select
@@ -834,6 +890,7 @@ __global__ void __cluster_dims__(kSmallCluster, 1, 1) __launch_bounds__(kSmallTh
             rec.fedges = fedges;
             rec.unvisited = unvisited;
             rec.probes = 0;
+            rec.la_found = 0;
             rec.strategy = XBFS_SF;
             rec.pad = 0;
             a.log[k] = rec;
@@ -925,16 +982,20 @@ __device__ __forceinline__ void grid_sync(unsigned* ctr, unsigned& epoch) {
     __syncthreads();
 }
 
+template <bool LA>
 union PersistSmem {
     TdSmem td;
-    BuSmem<kPersistThreads / 32> bu;
+    typename std::conditional<LA, BuSmemLa<kPersistThreads / 32>, BuSmem<kPersistThreads / 32>>::type bu;
 };
 
+// LA: the BU look-ahead variant (a separate instantiation, so the default kernel
+// carries none of its registers).
+template <bool LA>
 __global__ __launch_bounds__(kPersistThreads, kPersistBlocks) void k_persist(
     KArgs a, int* __restrict__ level, int* __restrict__ parent, const unsigned int* __restrict__ nonisolated,
     long long nonisolated_count) {
     extern __shared__ __align__(16) unsigned char dsm[];
-    PersistSmem& sm = *reinterpret_cast<PersistSmem*>(dsm);
+    PersistSmem<LA>& sm = *reinterpret_cast<PersistSmem<LA>*>(dsm);
     __shared__ SelState s;
     unsigned epoch = 0;
     unsigned* bar = &a.st->bar_count;
@@ -956,6 +1017,7 @@ __global__ __launch_bounds__(kPersistThreads, kPersistBlocks) void k_persist(
             a.st->qctr[(k + 2) % 3] = 0;
             a.st->qmax[(k + 2) % 3] = 0;
             a.st->acc_found[(k + 1) % 3] = a.st->acc_edges[(k + 1) % 3] = a.st->acc_probes[(k + 1) % 3] = 0;
+            a.st->acc_la_found[(k + 1) % 3] = a.st->acc_la_edges[(k + 1) % 3] = 0;
         }
         if (strat != XBFS_BU && !qvalid) {
             generate_body(a, k, 0);
@@ -968,11 +1030,15 @@ __global__ __launch_bounds__(kPersistThreads, kPersistBlocks) void k_persist(
             grid_sync(bar, epoch);
             ss_count_body(a, k);
         } else {
-            bu_body<kPersistThreads / 32>(a, &s.k, level, parent, sm.bu);
+            bu_body<kPersistThreads / 32, LA>(a, &s.k, level, parent, sm.bu, s.prefill);
         }
         grid_sync(bar, epoch);
         if (threadIdx.x == 0) select_step(a, s, blockIdx.x == 0, blockIdx.x == 0 ? globaltimer() : 0ull);
         __syncthreads();
+        if (LA && s.la_cf > 0) {    // look-ahead vertices of step k join F_{k+2} before step k+1
+            la_merge(a, s.k);
+            grid_sync(bar, epoch);
+        }
     }
     if (blockIdx.x == 0 && threadIdx.x == 0) sel_store(a.st, s);
 }
@@ -1222,28 +1288,28 @@ xbfs_status build_loop_graph(xbfs_graph* g, int* level, int* parent) {
     return XBFS_OK;
 }
 
-xbfs_status launch_persist(xbfs_graph* g, const KArgs& a, int* level, int* parent) {
-    static int occ[64];
-    static bool init[64] = {false};
-    const int dev = g->device & 63;
-    if (!init[dev]) {
-        XBFS_CUDA(g, cudaFuncSetAttribute(k_persist, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                          (int)sizeof(PersistSmem)));
+xbfs_status launch_persist(xbfs_graph* g, const KArgs& a, int* level, int* parent, bool lookahead) {
+    static int occ[2][64];
+    static bool init[2][64] = {{false}};
+    const int dev = g->device & 63, v = lookahead ? 1 : 0;
+    void* fn = lookahead ? (void*)k_persist<true> : (void*)k_persist<false>;
+    const size_t smem = lookahead ? sizeof(PersistSmem<true>) : sizeof(PersistSmem<false>);
+    if (!init[v][dev]) {
+        XBFS_CUDA(g, cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
         int o = 0;
-        XBFS_CUDA(g, cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, k_persist, kPersistThreads,
-                                                                   sizeof(PersistSmem)));
-        occ[dev] = o;
-        init[dev] = true;
+        XBFS_CUDA(g, cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, fn, kPersistThreads, smem));
+        occ[v][dev] = o;
+        init[v][dev] = true;
     }
-    if (occ[dev] < 1) return set_error(XBFS_ERR_UNSUPPORTED, "persistent driver: k_persist does not fit on an SM");
-    const int grid = g->num_sms * std::min(occ[dev], kPersistBlocks);
+    if (occ[v][dev] < 1) return set_error(XBFS_ERR_UNSUPPORTED, "persistent driver: k_persist does not fit on an SM");
+    const int grid = g->num_sms * std::min(occ[v][dev], kPersistBlocks);
     const unsigned int* noniso = g->nonisolated;
     long long nic = g->nonisolated_count;
     KArgs ka = a;
     ka.track_max = 0;   // no small-frontier mode inside the persistent kernel
     void* args[] = {&ka, &level, &parent, &noniso, &nic};
-    XBFS_CUDA(g, cudaLaunchCooperativeKernel((void*)k_persist, dim3(grid), dim3(kPersistThreads), args,
-                                             sizeof(PersistSmem), g->stream));
+    XBFS_CUDA(g, cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(kPersistThreads), args, smem,
+                                             g->stream));
     return XBFS_OK;
 }
 
@@ -1271,6 +1337,8 @@ static xbfs_status run_impl(xbfs_graph* g, int64_t source, int32_t* level, int32
     const bool host_only = (stats && stats->kernel_capacity > 0) || (o.plan && o.plan_len > 0);
     const bool use_persist = (o.driver == 0 || o.driver == 3) && !host_only;
     const bool use_graph = o.driver == 2 && !host_only;
+    if (o.lookahead && !use_persist)
+        return set_error(XBFS_ERR_INVALID_ARG, "lookahead needs the persistent driver (driver 0/3, no plan/profiling)");
     // selection parameters live in the device state
     {
         DevState hs;
@@ -1283,6 +1351,7 @@ static xbfs_status run_impl(xbfs_graph* g, int64_t source, int32_t* level, int32
         hs.source = source;
         hs.small_edges = std::min<long long>(std::max(o.small_edges, 0), kSmallEdgesMax);
         hs.mirror_host = (use_graph || use_persist) ? 0 : 1;
+        hs.lookahead = o.lookahead ? 1 : 0;
         XBFS_CUDA(g, cudaMemcpyAsync(g->st, &hs, sizeof(hs), cudaMemcpyHostToDevice, g->stream));
     }
     const Grids G = grids_for(g);
@@ -1291,7 +1360,7 @@ static xbfs_status run_impl(xbfs_graph* g, int64_t source, int32_t* level, int32
     P.st = stats;
     if (use_persist) {
         XBFS_CUDA(g, cudaEventRecord(g->ev0, g->stream));
-        XBFS_TRY(launch_persist(g, a, level, parent));
+        XBFS_TRY(launch_persist(g, a, level, parent, o.lookahead != 0));
         XBFS_CUDA(g, cudaEventRecord(g->ev1, g->stream));
     } else if (use_graph) {
         XBFS_TRY(build_loop_graph(g, level, parent));
@@ -1329,7 +1398,7 @@ static xbfs_status run_impl(xbfs_graph* g, int64_t source, int32_t* level, int32
         XBFS_TRY(P.finish());
         const int nl = std::min(hs.nlevels, std::min(stats->level_capacity, kLogCap));
         if (nl > 0 && (stats->strategy || stats->frontier_vertices || stats->frontier_edges ||
-                       stats->unvisited || stats->bu_probes || stats->level_ms)) {
+                       stats->unvisited || stats->bu_probes || stats->level_ms || stats->lookahead_found)) {
             LevelRec* rec = new LevelRec[nl];
             XBFS_CUDA(g, cudaMemcpy(rec, g->log, nl * sizeof(LevelRec), cudaMemcpyDeviceToHost));
             for (int i = 0; i < nl; ++i) {
@@ -1338,6 +1407,7 @@ static xbfs_status run_impl(xbfs_graph* g, int64_t source, int32_t* level, int32
                 if (stats->frontier_edges) stats->frontier_edges[i] = rec[i].fedges;
                 if (stats->unvisited) stats->unvisited[i] = rec[i].unvisited;
                 if (stats->bu_probes) stats->bu_probes[i] = rec[i].probes;
+                if (stats->lookahead_found) stats->lookahead_found[i] = rec[i].la_found;
                 if (stats->level_ms) {
                     const unsigned long long t0 = i ? rec[i - 1].t_ns : hs.t_start;
                     stats->level_ms[i] = (use_persist && rec[i].t_ns >= t0 && t0) ? (float)((rec[i].t_ns - t0) * 1e-6)

@@ -10,6 +10,7 @@ namespace xbfs {
 // starts at 0); col values and the frontier bitmap `cur` are GLOBAL.
 struct BuView {
     const unsigned int* cur;          // F_k, global bitmap
+    const unsigned int* nxt;          // F_{k+1} being written by this pass (look-ahead only)
     unsigned int* visited;            // owned words
     long long words;                  // owned words
     const unsigned long long* head;   // owned: deg << 32 | first stored neighbour
@@ -31,13 +32,34 @@ struct BuSmem {
     unsigned found[WARPS][kBuChunkWords];
 };
 
-// publish(w, vis, found_word): store the owned word w of F_{k+1} and update visited.
+// ... plus the look-ahead lists (kept out of the default kernels' shared memory).
+template <int WARPS>
+struct BuSmemLa : BuSmem<WARPS> {
+    int hlau[WARPS][kBuChunkWords * 32];   // F_{k+1} neighbour seen before a row went hard
+    unsigned la[WARPS][kBuChunkWords];     // look-ahead discoveries (level k+2)
+};
+
+// Look-ahead accumulators: vertices set to level k+2 by a BU pass.
+struct BuLa {
+    unsigned long long found = 0, edges = 0;
+};
+
+// publish(w, vis, found_word, la_word): store the owned word w of F_{k+1} (and of
+// the look-ahead set) and update visited.
 // Mutable state (visited, cur) is read through L2 (__ldcg): the persistent
 // driver runs every level inside one kernel, where L1 lines are not refreshed.
-template <int WARPS, class Publish>
-__device__ __forceinline__ void bu_chunks(const BuView& b, BuSmem<WARPS>& sm, Publish publish,
+//
+// LA ("since v7 is updated in this phase, v8, which
+// belongs to the next level, can be updated in this bottom-up"): a candidate whose
+// whole row holds no F_k vertex but some vertex already published into F_{k+1}
+// by this same pass is at level k+2 exactly (no neighbour at level <= k, one at
+// k+1: the exactness guard of reading C-9), with that neighbour as parent.  Only
+// published F_{k+1} words are seen (whole-word stores), so a set bit is always a
+// true level-(k+1) vertex; which candidates profit depends on the pass order.
+template <int WARPS, bool LA, class Smem, class Publish>
+__device__ __forceinline__ void bu_chunks(const BuView& b, Smem& sm, Publish publish,
                                           unsigned long long& found, unsigned long long& edges,
-                                          unsigned long long& probes, unsigned& fmax) {
+                                          unsigned long long& probes, unsigned& fmax, BuLa& la) {
     constexpr unsigned FULL = 0xffffffffu;
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
     const unsigned lt = (1u << lane) - 1u;
@@ -87,8 +109,21 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, BuSmem<WARPS>& sm, Pu
             const int total = __shfl_sync(FULL, incl, 31);
             int pos = incl - cnt;
             for (unsigned bits = cand; bits; bits &= bits - 1) s_list[wib][pos++] = (int)(w * 32 + __ffs(bits) - 1);
-            if (lane < kCW) s_found[wib][lane] = 0;
+            if (lane < kCW) {
+                s_found[wib][lane] = 0;
+                if constexpr (LA) sm.la[wib][lane] = 0;
+            }
             __syncwarp();
+            // a look-ahead discovery of v (level k+2) with parent pu (F_{k+1})
+            auto la_store = [&](int v, int pu, long long deg) {
+                if constexpr (LA) {
+                    b.level[v] = b.lvl + 1;
+                    b.parent[v] = pu;
+                    atomicOr(&sm.la[wib][(v >> 5) - c * kCW], 1u << (v & 31));
+                    la.found += 1;
+                    la.edges += (unsigned long long)deg;
+                }
+            };
             // 2. first probe of every candidate, kBuFirstIlp candidates per lane in flight:
             //    head[v] (deg << 32 | first stored neighbour) is a dense array read in
             //    candidate order, so a hit (the common case after the degree-desc
@@ -98,7 +133,7 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, BuSmem<WARPS>& sm, Pu
             for (int base = 0; base < total; base += 32 * kBuFirstIlp) {
                 int vv[kBuFirstIlp];
                 unsigned long long hv[kBuFirstIlp];
-                unsigned wd[kBuFirstIlp];
+                unsigned wd[kBuFirstIlp], wn[kBuFirstIlp];
     #pragma unroll
                 for (int g = 0; g < kBuFirstIlp; ++g) {
                     const int idx = base + g * 32 + lane;
@@ -110,6 +145,8 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, BuSmem<WARPS>& sm, Pu
                 for (int g = 0; g < kBuFirstIlp; ++g) {
                     const int fu = (int)(unsigned)hv[g];
                     wd[g] = vv[g] >= 0 ? __ldcg(b.cur + (fu >> 5)) : 0u;
+                    // look-ahead: a degree-1 miss needs its only neighbour's F_{k+1} bit
+                    wn[g] = (LA && vv[g] >= 0 && (hv[g] >> 32) == 1) ? __ldcg(b.nxt + (fu >> 5)) : 0u;
                 }
                 __syncwarp();   // every read of this round is done before the in-place compaction
     #pragma unroll
@@ -129,6 +166,7 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, BuSmem<WARPS>& sm, Pu
                             probes += 1;
                         } else if (d == 1) {
                             probes += 1;
+                            if (LA && ((wn[g] >> (fu & 31)) & 1u)) la_store(v, fu, 1);
                         } else {
                             miss = true;
                         }
@@ -140,9 +178,10 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, BuSmem<WARPS>& sm, Pu
             }
             __syncwarp();
             // 3. the misses: lane-per-candidate, kBuBatch arcs per step in stored
-            //    order from the second arc on; a lane that finishes takes the next
-            //    candidate, so lanes stay busy.
-            int v = -1, nxt = 0, nhard = 0;
+            //    order from the second arc on (look-ahead: from the first, whose
+            //    F_{k+1} bit pass 1 did not read); a lane that finishes takes the
+            //    next candidate, so lanes stay busy.
+            int v = -1, nxt = 0, nhard = 0, lau = -1;
             long long rs = 0, re = 0, p = 0;
             for (;;) {
                 const unsigned need = __ballot_sync(FULL, v < 0);
@@ -152,7 +191,8 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, BuSmem<WARPS>& sm, Pu
                         v = s_list[wib][idx];
                         rs = b.row_ptr[v];
                         re = b.row_ptr[v + 1];
-                        p = rs + 1;
+                        p = LA ? rs : rs + 1;
+                        lau = -1;
                     }
                 }
                 nxt += __popc(need);
@@ -161,15 +201,23 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, BuSmem<WARPS>& sm, Pu
                 if (v >= 0) {
                     const long long end = min(re, p + kBuBatch);
                     int u[kBuBatch];
-                    unsigned wd[kBuBatch];
+                    unsigned wd[kBuBatch], wn[kBuBatch];
     #pragma unroll
                     for (int j = 0; j < kBuBatch; ++j) u[j] = (p + j < end) ? __ldg(b.col + p + j) : -1;
     #pragma unroll
-                    for (int j = 0; j < kBuBatch; ++j) wd[j] = u[j] >= 0 ? __ldcg(b.cur + (u[j] >> 5)) : 0u;
+                    for (int j = 0; j < kBuBatch; ++j) {
+                        wd[j] = u[j] >= 0 ? __ldcg(b.cur + (u[j] >> 5)) : 0u;
+                        wn[j] = (LA && lau < 0 && u[j] >= 0) ? __ldcg(b.nxt + (u[j] >> 5)) : 0u;
+                    }
                     int hit = -1;
     #pragma unroll
                     for (int j = kBuBatch - 1; j >= 0; --j)
                         if (u[j] >= 0 && ((wd[j] >> (u[j] & 31)) & 1u)) hit = j;   // first hit in row order
+                    if (LA && lau < 0) {
+    #pragma unroll
+                        for (int j = kBuBatch - 1; j >= 0; --j)
+                            if (u[j] >= 0 && ((wn[j] >> (u[j] & 31)) & 1u)) lau = u[j];
+                    }
                     if (hit >= 0) {
                         int pu = u[0];
     #pragma unroll
@@ -184,6 +232,7 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, BuSmem<WARPS>& sm, Pu
                         v = -1;
                     } else if (end == re) {
                         probes += (unsigned long long)(re - rs);
+                        if (LA && lau >= 0) la_store(v, lau, re - rs);
                         v = -1;
                     } else if (re - end > kBuHardMin) {
                         to_hard = true;
@@ -196,6 +245,7 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, BuSmem<WARPS>& sm, Pu
                     const int hi = nhard + __popc(hm & lt);
                     s_hard[wib][hi] = v;
                     s_hoff[wib][hi] = (int)(p + kBuBatch - rs);
+                    if constexpr (LA) sm.hlau[wib][hi] = lau;
                     v = -1;
                 }
                 nhard += __popc(hm);
@@ -205,6 +255,8 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, BuSmem<WARPS>& sm, Pu
             for (int h = 0; h < nhard; ++h) {
                 const int hv = s_hard[wib][h];
                 const long long hrs = b.row_ptr[hv], hre = b.row_ptr[hv + 1];
+                int hl = -1;
+                if constexpr (LA) hl = sm.hlau[wib][h];
                 bool hit_any = false;
                 for (long long base = hrs + s_hoff[wib][h]; base < hre; base += 32) {
                     const long long pp = base + lane;
@@ -225,13 +277,23 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, BuSmem<WARPS>& sm, Pu
                         hit_any = true;
                         break;
                     }
+                    if (LA && hl < 0) {
+                        const bool nb = u >= 0 && ((__ldcg(b.nxt + (u >> 5)) >> (u & 31)) & 1u);
+                        const unsigned mn = __ballot_sync(FULL, nb);
+                        if (mn) hl = __shfl_sync(FULL, u, __ffs(mn) - 1);
+                    }
                 }
-                if (!hit_any && lane == 0) probes += (unsigned long long)(hre - hrs);
+                if (!hit_any && lane == 0) {
+                    probes += (unsigned long long)(hre - hrs);
+                    if (LA && hl >= 0) la_store(hv, hl, hre - hrs);
+                }
             }
             __syncwarp();
             if (own) {
                 const unsigned f = s_found[wib][lane];
-                if (f) publish(w, vis, f);   // zero words are already zero in every replica
+                unsigned lf = 0u;
+                if constexpr (LA) lf = sm.la[wib][lane];
+                if (f | lf) publish(w, vis, f, lf);   // zero words are already zero in every replica
             }
             __syncwarp();
         }

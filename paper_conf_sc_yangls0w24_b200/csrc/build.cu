@@ -170,7 +170,7 @@ xbfs_status alloc_work(xbfs_graph* g) {
     const long long n = g->n, words = (n + 31) / 32;
     g->tiles_cap = g->arcs / kTile + 4;
     XBFS_CUDA(g, cudaMalloc(&g->visited, words * sizeof(unsigned int)));
-    XBFS_CUDA(g, cudaMalloc(&g->fb, 3 * ((words + 31) / 32 * 32) * sizeof(unsigned int)));
+    XBFS_CUDA(g, cudaMalloc(&g->fb, 4 * ((words + 31) / 32 * 32) * sizeof(unsigned int)));
     XBFS_CUDA(g, cudaMalloc(&g->qv, 3 * n * sizeof(int)));
     XBFS_CUDA(g, cudaMalloc(&g->qoff, 3 * n * sizeof(long long)));
     XBFS_CUDA(g, cudaMalloc(&g->qdelta, 3 * n * sizeof(long long)));

@@ -43,6 +43,7 @@ constexpr int kPersistBlocks = 2;    // ... CTAs per SM (64 registers per thread
 
 struct LevelRec {
     long long fsize, fedges, unvisited, probes;
+    long long la_found;        // vertices this step set to level k+2 (BU look-ahead)
     int strategy, pad;
     unsigned long long t_ns;   // %globaltimer at the end of the level (persistent driver; 0 otherwise)
 };
@@ -69,6 +70,7 @@ struct DevState {
     long long unvisited;         // U_k (non-isolated, unvisited)
     unsigned long long acc_found[3], acc_edges[3], acc_probes[3];  // BU / SS-count accumulators:
                                  // level k adds into slot k%3; slot (k+1)%3 is zeroed before level k+1
+    unsigned long long acc_la_found[3], acc_la_edges[3];  // BU look-ahead (level k+2) discoveries, same slots
     long long reached, arcs_traversed;
     unsigned int launches;       // library kernels launched (device-counted)
     int nlevels;
@@ -80,7 +82,7 @@ struct DevState {
     int advanced;                // k_small already advanced the level state: k_select only mirrors it
     int prev_small;              // level k-1 was a small SF level (small-mode entry gate)
     int mirror_host;             // host-loop driver: mirror the level state into HostCtl
-    int pad2_;
+    int lookahead;               // BU look-ahead (persistent driver)
     unsigned long long t_start;  // %globaltimer after init + seed (persistent driver)
     // persistent driver: grid-barrier arrival counter, alone on its 128-byte line
     // (zeroed with the rest of the state before every run)
@@ -97,6 +99,7 @@ struct KArgs {
     const unsigned long long* head;  // per vertex: deg << 32 | first stored neighbour (BU first probe)
     unsigned int* visited;
     unsigned int* fb[3];
+    unsigned int* la;       // look-ahead bitmap: level-(k+2) vertices found by BU step k
     int* qv[3];
     long long* qoff[3];
     long long* qdelta[3];
@@ -130,7 +133,7 @@ struct xbfs_graph {
     long long nonisolated_count = 0;
     // BFS work state
     unsigned int* visited = nullptr;
-    unsigned int* fb = nullptr;          // 3 * words
+    unsigned int* fb = nullptr;          // 4 * stride words: 3 frontier maps + the look-ahead map
     int* qv = nullptr;                   // 3 * N (queue of F_k in buffer k%3)
     long long* qoff = nullptr;           // 3 * N
     long long* qdelta = nullptr;         // 3 * N

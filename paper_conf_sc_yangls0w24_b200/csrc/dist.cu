@@ -123,6 +123,7 @@ __global__ __launch_bounds__(kBuThreads, 4) void k_bu(DArgs a, int k) {
         a.fb[(k + 2) % 3][w] = 0;
     BuView b;
     b.cur = a.fb[k % 3];
+    b.nxt = nullptr;
     b.visited = a.vis;
     b.words = a.cw;
     b.head = a.head;
@@ -132,13 +133,14 @@ __global__ __launch_bounds__(kBuThreads, 4) void k_bu(DArgs a, int k) {
     b.parent = a.parent;
     b.lvl = k + 1;
     __shared__ BuSmem<kBuThreads / 32> sm;
-    bu_chunks<kBuThreads / 32>(b, sm, [&](long long w, unsigned vis, unsigned f) {
+    BuLa la_unused;
+    bu_chunks<kBuThreads / 32, false>(b, sm, [&](long long w, unsigned vis, unsigned f, unsigned) {
         publish_word(a, slot, w, f);
         if (f) {
             a.vis[w] = vis | f;
             for (unsigned bits = f; bits; bits &= bits - 1) m += (unsigned long long)a.tcount[w * 32 + __ffs(bits) - 1];
         }
-    }, found, edges, probes, fmax);
+    }, found, edges, probes, fmax, la_unused);
     for (int o = 16; o; o >>= 1) {
         found += __shfl_xor_sync(FULL, found, o);
         edges += __shfl_xor_sync(FULL, edges, o);

@@ -42,7 +42,7 @@ class RunOpts(ctypes.Structure):
     _fields_ = [("alpha", ctypes.c_double), ("grow", ctypes.c_double), ("ratio_min", ctypes.c_double),
                 ("bu_stay", ctypes.c_double), ("force_strategy", ctypes.c_int32), ("driver", ctypes.c_int32),
                 ("small_edges", ctypes.c_int32), ("plan_len", ctypes.c_int32),
-                ("plan", ctypes.POINTER(ctypes.c_int8))]
+                ("plan", ctypes.POINTER(ctypes.c_int8)), ("lookahead", ctypes.c_int32)]
 
 
 class RunStats(ctypes.Structure):
@@ -55,7 +55,8 @@ class RunStats(ctypes.Structure):
                 ("bu_probes", ctypes.POINTER(ctypes.c_int64)),
                 ("kernel_capacity", ctypes.c_int32), ("num_kernels", ctypes.c_int32),
                 ("kernel_id", ctypes.POINTER(ctypes.c_int32)), ("kernel_level", ctypes.POINTER(ctypes.c_int32)),
-                ("kernel_ms", ctypes.POINTER(ctypes.c_float)), ("level_ms", ctypes.POINTER(ctypes.c_float))]
+                ("kernel_ms", ctypes.POINTER(ctypes.c_float)), ("level_ms", ctypes.POINTER(ctypes.c_float)),
+                ("lookahead_found", ctypes.POINTER(ctypes.c_int64))]
 
 
 #: kernel ids of RunStats.kernel_id (XBFS_K_* in include/xbfs.h)
@@ -175,6 +176,7 @@ class Stats:
     bu_probes: list = field(default_factory=list)
     kernels: list = field(default_factory=list)   # (name, level, ms) when profiled
     level_ms: list = field(default_factory=list)  # device ms per level (persistent driver)
+    lookahead_found: list = field(default_factory=list)  # level-(k+2) vertices set by BU step k
 
 
 class _StatsBuf:
@@ -186,6 +188,7 @@ class _StatsBuf:
         self.un = np.zeros(cap, np.int64)
         self.pr = np.zeros(cap, np.int64)
         self.lms = np.zeros(cap, np.float32)
+        self.laf = np.zeros(cap, np.int64)
         self.c = RunStats()
         self.c.level_capacity = cap
         P = lambda a, t: a.ctypes.data_as(ctypes.POINTER(t))
@@ -195,6 +198,7 @@ class _StatsBuf:
         self.c.unvisited = P(self.un, ctypes.c_int64)
         self.c.bu_probes = P(self.pr, ctypes.c_int64)
         self.c.level_ms = P(self.lms, ctypes.c_float)
+        self.c.lookahead_found = P(self.laf, ctypes.c_int64)
         self.kcap = kernel_cap
         if kernel_cap:
             self.kid = np.zeros(kernel_cap, np.int32)
@@ -213,15 +217,16 @@ class _StatsBuf:
                      self.un[:nl].tolist(), self.pr[:nl].tolist(),
                      [(KERNEL_NAMES[int(self.kid[i])], int(self.klv[i]), float(self.kms[i]))
                       for i in range(min(c.num_kernels, self.kcap))] if self.kcap else [],
-                     self.lms[:nl].tolist())
+                     self.lms[:nl].tolist(), self.laf[:nl].tolist())
 
 
 def make_run_opts(alpha=None, grow=None, ratio_min=None, bu_stay=None, force_strategy=None, driver=None,
-                  small_edges=None, plan=None) -> RunOpts:
+                  small_edges=None, plan=None, lookahead=None) -> RunOpts:
     """plan: sequence of per-level strategies (-1 = selector, 0 SF, 1 SS, 2 BU)."""
     o = xbfs_run_opts_default()
     for k, v in dict(alpha=alpha, grow=grow, ratio_min=ratio_min, bu_stay=bu_stay,
-                     force_strategy=force_strategy, driver=driver, small_edges=small_edges).items():
+                     force_strategy=force_strategy, driver=driver, small_edges=small_edges,
+                     lookahead=lookahead).items():
         if v is not None:
             setattr(o, k, v)
     if plan is not None and len(plan):

@@ -311,3 +311,41 @@ def test_unaligned_output_arrays(xb):
             assert oracle.validate(og, src, dst, int(root), lv, pa) == 0
             assert int(lbuf[0]) == 7 and int(pbuf[0]) == 7
     g.close()
+
+
+@pytest.mark.parametrize("graph", ["kron", "grid", "hub"])
+def test_bu_lookahead(xb, graph):
+    """BU look-ahead: a BU step also settles level k+2
+    vertices whose whole row misses F_k but hits a vertex this pass already put
+    into F_{k+1}.  Levels stay bit-exact, parents valid, per-level frontier sizes
+    exact (the look-ahead vertices are merged into F_{k+2} before step k+1, for
+    a BU, SS or SF step k+1 alike), and the look-ahead does fire."""
+    if graph == "kron":
+        src, dst, n = synth.kronecker(15, seed=6)
+        roots = synth.roots(n, src, dst, 4, root_seed=9)
+    elif graph == "grid":
+        src, dst, n = synth.grid(40, 30, seed=2)
+        roots = [0, n // 2, n - 1]
+    else:
+        rng = np.random.default_rng(3)
+        n = 6000
+        e = np.concatenate([np.stack([np.zeros(3000, np.int64), rng.integers(1, n, 3000)], 1),
+                            rng.integers(0, n, (15000, 2))]).astype(np.uint32)
+        src, dst = e[:, 0].copy(), e[:, 1].copy()
+        roots = [0, 1, 5999]
+    og = oracle.build_csr(n, src, dst)
+    g = xb.Graph(_dev(src), _dev(dst), n)
+    fired = 0
+    for root in roots:
+        for opts in (dict(lookahead=1), dict(lookahead=1, force_strategy=2), dict(lookahead=1, alpha=0.005),
+                     dict(lookahead=1, alpha=0.3, bu_stay=0.0), dict(lookahead=1, driver=3, bu_stay=8.0)):
+            st = _check_run(g, og, src, dst, root, **opts)
+            assert all(x == 0 for k, x in enumerate(st.lookahead_found) if st.strategy[k] != 2)
+            fired += sum(st.lookahead_found)
+    assert fired > 0
+    # without the option nothing is set ahead
+    st = _check_run(g, og, src, dst, roots[0], force_strategy=2)
+    assert sum(st.lookahead_found) == 0
+    with pytest.raises(xb.XbfsError):
+        g.run(int(roots[0]), lookahead=1, driver=1)
+    g.close()
