@@ -349,3 +349,21 @@ def test_bu_lookahead(xb, graph):
     with pytest.raises(xb.XbfsError):
         g.run(int(roots[0]), lookahead=1, driver=1)
     g.close()
+
+
+@pytest.mark.parametrize("cfg", ["s24", "grid"])
+def test_bench_workload_full_size(xb, cfg):
+    """The exact graphs and roots bench.py times (BASELINE configs 3 and 5 at full
+    size: Kronecker s24 ef16 seed 1, 16.8 M vertices / 521 M arcs; the 4096^2
+    grid), in bench's launch configuration (persistent driver, default options):
+    levels bit-exact against the oracle's serial BFS of the whole graph, parents
+    Graph500-valid, per-level counters exact."""
+    import bench
+    src, dst, n = bench.make_graph(cfg, pinned=False)
+    og = oracle.build_csr(n, src, dst)
+    g = xb.Graph(_dev(src), _dev(dst), n)
+    roots = bench.pick_roots(cfg, n, src, dst, 4 if cfg == "s24" else 2)
+    for root in roots:
+        st = _check_run(g, og, src, dst, root)
+        assert st.kernel_launches == 1          # one cooperative launch per BFS
+    g.close()
