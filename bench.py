@@ -43,6 +43,7 @@ CONFIGS = {
     "s22": dict(kind="kron", scale=22, edgefactor=16),
     "s24": dict(kind="kron", scale=24, edgefactor=16),
     "s25": dict(kind="kron", scale=25, edgefactor=16),
+    "s27": dict(kind="kron", scale=27, edgefactor=16),   # BASELINE config 4's graph (p = 1 point)
     "grid": dict(kind="grid", width=4096, height=4096),
 }
 GRAPH_SEED, ROOT_SEED = 1, 2
