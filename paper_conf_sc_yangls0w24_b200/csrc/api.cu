@@ -36,6 +36,8 @@ xbfs::KArgs xbfs_graph::kargs() const {
     a.level = nullptr;
     a.parent = nullptr;
     a.head = head;
+    a.head32 = head32;
+    a.idbits = idbits;
     a.visited = visited;
     const long long stride = (words + 31) / 32 * 32;  // 128-byte aligned bitmaps (uint4 access)
     for (int i = 0; i < 3; ++i) a.fb[i] = fb + i * stride;
@@ -114,7 +116,7 @@ void xbfs_destroy(xbfs_graph* g) {
     g->drop_loops();
     void* dev[] = {g->row_ptr, g->col, g->tcount, g->nonisolated, g->visited, g->fb, g->qv,
                    g->qoff, g->qdelta, g->tile_first, g->st, g->log, g->red_scratch,
-                   g->scratch_level, g->scratch_parent, g->head};
+                   g->scratch_level, g->scratch_parent, g->head, g->head32};
     for (void* p : dev)
         if (p) cudaFree(p);
     if (g->hctl) cudaFreeHost(g->hctl);

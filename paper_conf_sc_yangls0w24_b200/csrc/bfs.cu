@@ -37,6 +37,11 @@ namespace xbfs {
 
 constexpr unsigned FULL = 0xffffffffu;
 
+// BU first probe from the 4-byte head32[] (1) or the 8-byte head[] (0; A/B only)
+#ifndef XBFS_BU_H32
+#define XBFS_BU_H32 1
+#endif
+
 __device__ __forceinline__ void count_launch(DevState* st) {
     if (blockIdx.x == 0 && threadIdx.x == 0) atomicAdd(&st->launches, 1u);
 }
@@ -660,6 +665,8 @@ __device__ __forceinline__ void bu_body(const KArgs& a, const int* kp, int* __re
     b.visited = a.visited;
     b.words = a.words;
     b.head = a.head;
+    b.head32 = a.head32;
+    b.idbits = a.idbits;
     b.row_ptr = a.row_ptr;
     b.col = a.col;
     b.level = level;
@@ -667,7 +674,7 @@ __device__ __forceinline__ void bu_body(const KArgs& a, const int* kp, int* __re
     b.lvl = lvl;
     // prefill: F_{k+1} already holds look-ahead vertices of step k-1 (OR into it)
     const bool pf = LA && prefill;
-    bu_chunks<WARPS, LA>(b, sm, [&](long long w, unsigned vis, unsigned f, unsigned lf) {
+    bu_chunks<WARPS, LA, XBFS_BU_H32>(b, sm, [&](long long w, unsigned vis, unsigned f, unsigned lf) {
         if (pf) f |= __ldcg(next + w);
         if (f) next[w] = f;
         a.visited[w] = vis | f | lf;

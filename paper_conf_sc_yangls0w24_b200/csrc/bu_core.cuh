@@ -14,6 +14,8 @@ struct BuView {
     unsigned int* visited;            // owned words
     long long words;                  // owned words
     const unsigned long long* head;   // owned: deg << 32 | first stored neighbour
+    const unsigned* head32;           // single GPU: min(deg, dmax) << idbits | first neighbour (H32)
+    int idbits;
     const long long* row_ptr;         // owned rows
     const int* col;
     int* level;                       // owned
@@ -56,7 +58,11 @@ struct BuLa {
 // k+1: the exactness guard of reading C-9), with that neighbour as parent.  Only
 // published F_{k+1} words are seen (whole-word stores), so a set bit is always a
 // true level-(k+1) vertex; which candidates profit depends on the pass order.
-template <int WARPS, bool LA, class Smem, class Publish>
+//
+// H32 (single GPU): the first probe reads the 4-byte head32[] word; a hit whose
+// degree field saturated (deg >= dmax) is queued for pass 3 as ~v, where one
+// row_ptr pair read (overlapping the misses' own) gives the degree for edgesF.
+template <int WARPS, bool LA, bool H32, class Smem, class Publish>
 __device__ __forceinline__ void bu_chunks(const BuView& b, Smem& sm, Publish publish,
                                           unsigned long long& found, unsigned long long& edges,
                                           unsigned long long& probes, unsigned& fmax, BuLa& la) {
@@ -130,6 +136,8 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, Smem& sm, Publish pub
             //    re-arrangement) never touches row_ptr or col.  Misses with more
             //    arcs are compacted in place at the front of s_list.
             int nmiss = 0;
+            const unsigned idmask = H32 ? (b.idbits >= 32 ? 0xffffffffu : ((1u << b.idbits) - 1u)) : 0u;
+            const unsigned dmax = H32 ? (b.idbits >= 32 ? 0u : (0xffffffffu >> b.idbits)) : 0u;
             for (int base = 0; base < total; base += 32 * kBuFirstIlp) {
                 int vv[kBuFirstIlp];
                 unsigned long long hv[kBuFirstIlp];
@@ -139,8 +147,18 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, Smem& sm, Publish pub
                     const int idx = base + g * 32 + lane;
                     vv[g] = idx < total ? s_list[wib][idx] : -1;
                 }
+                if constexpr (H32) {
+                    // unpack to the 64-bit head layout (deg << 32 | first); a saturated
+                    // degree stays dmax (>= 2) and is resolved in pass 3 on a hit
     #pragma unroll
-                for (int g = 0; g < kBuFirstIlp; ++g) hv[g] = vv[g] >= 0 ? __ldg(b.head + vv[g]) : 0ull;
+                    for (int g = 0; g < kBuFirstIlp; ++g) {
+                        const unsigned h = vv[g] >= 0 ? __ldg(b.head32 + vv[g]) : 0u;
+                        hv[g] = ((unsigned long long)(b.idbits >= 32 ? 0u : (h >> b.idbits)) << 32) | (h & idmask);
+                    }
+                } else {
+    #pragma unroll
+                    for (int g = 0; g < kBuFirstIlp; ++g) hv[g] = vv[g] >= 0 ? __ldg(b.head + vv[g]) : 0ull;
+                }
     #pragma unroll
                 for (int g = 0; g < kBuFirstIlp; ++g) {
                     const int fu = (int)(unsigned)hv[g];
@@ -160,11 +178,15 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, Smem& sm, Publish pub
                             b.level[v] = b.lvl;
                             b.parent[v] = fu;
                             atomicOr(&s_found[wib][(v >> 5) - c * kCW], 1u << (v & 31));
-                            edges += (unsigned long long)d;
-                            fmax = max(fmax, (unsigned)d);
+                            if (!H32 || (unsigned)d < dmax) {
+                                edges += (unsigned long long)d;
+                                fmax = max(fmax, (unsigned)d);
+                            } else {
+                                miss = true;   // degree-only entry for pass 3 (stored as ~v)
+                            }
                             ++found;
                             probes += 1;
-                        } else if (d == 1) {
+                        } else if (d == 1 && (!H32 || dmax > 1)) {
                             probes += 1;
                             if (LA && ((wn[g] >> (fu & 31)) & 1u)) la_store(v, fu, 1);
                         } else {
@@ -172,7 +194,11 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, Smem& sm, Publish pub
                         }
                     }
                     const unsigned mm = __ballot_sync(FULL, miss);
-                    if (miss) s_list[wib][nmiss + __popc(mm & lt)] = v;
+                    if (miss) {
+                        // H32: a hit with a saturated degree goes in as ~v (degree only)
+                        const bool deg_only = H32 && ((wd[g] >> ((int)(unsigned)hv[g] & 31)) & 1u);
+                        s_list[wib][nmiss + __popc(mm & lt)] = deg_only ? ~v : v;
+                    }
                     nmiss += __popc(mm);
                 }
             }
@@ -189,14 +215,22 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, Smem& sm, Publish pub
                     const int idx = nxt + __popc(need & lt);
                     if (idx < nmiss) {
                         v = s_list[wib][idx];
-                        rs = b.row_ptr[v];
-                        re = b.row_ptr[v + 1];
-                        p = LA ? rs : rs + 1;
-                        lau = -1;
+                        if (H32 && v < 0) {          // found at the first probe; its degree only
+                            const int u0 = ~v;
+                            const long long dd = b.row_ptr[u0 + 1] - b.row_ptr[u0];
+                            edges += (unsigned long long)dd;
+                            fmax = max(fmax, (unsigned)dd);
+                            v = -1;
+                        } else {
+                            rs = b.row_ptr[v];
+                            re = b.row_ptr[v + 1];
+                            p = LA ? rs : rs + 1;
+                            lau = -1;
+                        }
                     }
                 }
                 nxt += __popc(need);
-                if (!__any_sync(FULL, v >= 0)) break;
+                if (!__any_sync(FULL, v >= 0) && nxt >= nmiss) break;   // (degree-only entries leave v < 0)
                 bool to_hard = false;
                 if (v >= 0) {
                     const long long end = min(re, p + kBuBatch);

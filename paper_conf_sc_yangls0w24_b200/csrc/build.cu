@@ -101,12 +101,19 @@ __global__ __launch_bounds__(kB) void k_degree_facts(const long long* __restrict
 
 // head[v] = deg(v) << 32 | first stored neighbour: the bottom-up first probe reads
 // this dense array in candidate order instead of a random sector of col.
+// head32[v] = min(deg(v), dmax) << idbits | first stored neighbour, dmax =
+// 2^(32 - idbits) - 1 meaning "deg >= dmax, read row_ptr": the single-GPU BU
+// first probe reads 4 bytes per candidate instead of 8 (idbits = bitlen(N-1)).
 __global__ __launch_bounds__(kB) void k_head(const long long* __restrict__ row_ptr, const int* __restrict__ col,
-                                             long long n, unsigned long long* __restrict__ head) {
+                                             long long n, unsigned long long* __restrict__ head,
+                                             unsigned* __restrict__ head32, int idbits) {
+    const unsigned dmax = idbits >= 32 ? 0u : (0xffffffffu >> idbits);
     for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < n;
          v += (long long)gridDim.x * blockDim.x) {
         const long long rs = row_ptr[v], d = row_ptr[v + 1] - rs;
         head[v] = ((unsigned long long)d << 32) | (d > 0 ? (unsigned)col[rs] : 0xffffffffu);
+        const unsigned dc = d < (long long)dmax ? (unsigned)d : dmax;
+        head32[v] = (idbits >= 32 ? 0u : (dc << idbits)) | (d > 0 ? (unsigned)col[rs] : 0u);
     }
 }
 
@@ -321,7 +328,9 @@ extern "C" xbfs_status xbfs_build_csr(const void* src, const void* dst, int64_t 
     g->nonisolated_count = (long long)facts[0];
     g->max_deg = (int)facts[1];
     XBFS_CUDA(g, cudaMalloc(&g->head, n * sizeof(unsigned long long)));
-    k_head<<<grid_for(n), kB, 0, g->stream>>>(g->row_ptr, g->col, n, g->head);
+    XBFS_CUDA(g, cudaMalloc(&g->head32, std::max<long long>(n, 1) * sizeof(unsigned)));
+    g->idbits = std::max(1, bitlen((unsigned long long)(n - 1)));
+    k_head<<<grid_for(n), kB, 0, g->stream>>>(g->row_ptr, g->col, n, g->head, g->head32, g->idbits);
     XBFS_CUDA(g, cudaGetLastError());
     if ((unsigned long long)arcs >= (1ull << g->dbits))
         return set_error(XBFS_ERR_INVALID_ARG, "graph too large for the packed queue counter");
@@ -368,7 +377,7 @@ extern "C" xbfs_status xbfs_reorder(xbfs_graph* g, int32_t mode) {
     }
     cudaFree(k0);
     cudaFree(k1);
-    k_head<<<grid_for(n), kB, 0, g->stream>>>(g->row_ptr, g->col, n, g->head);
+    k_head<<<grid_for(n), kB, 0, g->stream>>>(g->row_ptr, g->col, n, g->head, g->head32, g->idbits);
     XBFS_CUDA(g, cudaGetLastError());
     XBFS_CUDA(g, cudaStreamSynchronize(g->stream));
     // the BFS graph (if any) captured the old col pointer

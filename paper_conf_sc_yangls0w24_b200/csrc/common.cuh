@@ -96,7 +96,9 @@ struct KArgs {
     const int* col;
     int* level;
     int* parent;
-    const unsigned long long* head;  // per vertex: deg << 32 | first stored neighbour (BU first probe)
+    const unsigned long long* head;  // per vertex: deg << 32 | first stored neighbour
+    const unsigned* head32;          // per vertex: min(deg, dmax) << idbits | first neighbour (BU first probe)
+    int idbits;                      // bits of a vertex id in head32 (bitlen(N-1))
     unsigned int* visited;
     unsigned int* fb[3];
     unsigned int* la;       // look-ahead bitmap: level-(k+2) vertices found by BU step k
@@ -130,6 +132,8 @@ struct xbfs_graph {
     int* tcount = nullptr;
     unsigned int* nonisolated = nullptr;
     unsigned long long* head = nullptr;  // deg << 32 | col[row_ptr[v]] (rebuilt by every reorder)
+    unsigned* head32 = nullptr;          // the same in 4 bytes (degree capped, see k_head)
+    int idbits = 32;
     long long nonisolated_count = 0;
     // BFS work state
     unsigned int* visited = nullptr;

@@ -127,6 +127,8 @@ __global__ __launch_bounds__(kBuThreads, 4) void k_bu(DArgs a, int k) {
     b.visited = a.vis;
     b.words = a.cw;
     b.head = a.head;
+    b.head32 = nullptr;
+    b.idbits = 32;
     b.row_ptr = a.row_ptr;
     b.col = a.col;
     b.level = a.level;
@@ -134,7 +136,7 @@ __global__ __launch_bounds__(kBuThreads, 4) void k_bu(DArgs a, int k) {
     b.lvl = k + 1;
     __shared__ BuSmem<kBuThreads / 32> sm;
     BuLa la_unused;
-    bu_chunks<kBuThreads / 32, false>(b, sm, [&](long long w, unsigned vis, unsigned f, unsigned) {
+    bu_chunks<kBuThreads / 32, false, false>(b, sm, [&](long long w, unsigned vis, unsigned f, unsigned) {
         publish_word(a, slot, w, f);
         if (f) {
             a.vis[w] = vis | f;
