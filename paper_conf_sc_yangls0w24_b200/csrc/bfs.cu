@@ -408,15 +408,28 @@ struct TdSmem {
     int v[kTile + 1];
 };
 
+#ifndef XBFS_SF_PRECHECK_MIN
+#define XBFS_SF_PRECHECK_MIN 65536
+#endif
+constexpr long long kSfPrecheckMin = XBFS_SF_PRECHECK_MIN;   // edgesF_k above which SF probes before claiming
+
 template <int MODE, int THREADS>
 __device__ __forceinline__ void td_expand_body(const KArgs& a, int k, int* __restrict__ level,
-                                               int* __restrict__ parent, TdSmem& sm) {
+                                               int* __restrict__ parent, TdSmem& sm, long long Fs = -1,
+                                               long long Ts = -1) {
     clear_stale(a, k);
     const int in = k % 3, ob = (k + 1) % 3;
-    const unsigned long long q = __ldcg(&a.st->qctr[k % 3]);
-    const long long F = (long long)(q >> a.dbits);
-    const long long T = (long long)(q & ((1ull << a.dbits) - 1ull));
+    long long F = Fs, T = Ts;   // |F_k|, edgesF_k: from the caller's selector state when it has them
+    if (F < 0) {
+        const unsigned long long q = __ldcg(&a.st->qctr[k % 3]);
+        F = (long long)(q >> a.dbits);
+        T = (long long)(q & ((1ull << a.dbits) - 1ull));
+    }
     if (F == 0 || T == 0) return;
+    // small scan-free levels claim with the atomic directly (one round trip less
+    // per arc chain); large ones probe first so that arcs to visited vertices,
+    // the majority there, cost no atomic
+    const bool precheck = MODE != XBFS_SF || T > kSfPrecheckMin;
     const long long ntiles = (T + kTile - 1) / kTile;
     const int* __restrict__ qv = a.qv[in];
     const long long* __restrict__ qoff = a.qoff[in];
@@ -468,7 +481,7 @@ __device__ __forceinline__ void td_expand_body(const KArgs& a, int k, int* __res
             }
         }
 #pragma unroll
-        for (int i = 0; i < R; ++i) vis[i] = valid[i] ? __ldcg(visited + (v[i] >> 5)) : FULL;
+        for (int i = 0; i < R; ++i) vis[i] = !valid[i] ? FULL : (precheck ? __ldcg(visited + (v[i] >> 5)) : 0u);
         if (MODE == XBFS_SF) {
             unsigned old[R];
 #pragma unroll
@@ -1031,9 +1044,9 @@ __global__ __launch_bounds__(kPersistThreads, kPersistBlocks) void k_persist(
             grid_sync(bar, epoch);
         }
         if (strat == XBFS_SF) {
-            td_expand_body<XBFS_SF, kPersistThreads>(a, k, level, parent, sm.td);
+            td_expand_body<XBFS_SF, kPersistThreads>(a, k, level, parent, sm.td, s.fsize, s.fedges);
         } else if (strat == XBFS_SS) {
-            td_expand_body<XBFS_SS, kPersistThreads>(a, k, level, parent, sm.td);
+            td_expand_body<XBFS_SS, kPersistThreads>(a, k, level, parent, sm.td, s.fsize, s.fedges);
             grid_sync(bar, epoch);
             ss_count_body(a, k);
         } else {
