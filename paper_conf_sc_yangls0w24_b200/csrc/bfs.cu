@@ -269,7 +269,7 @@ __global__ void k_seed(KArgs a, int* level, int* parent, long long nonisolated_c
 // The level state the selector evolves (one copy per CTA in the persistent
 // driver, where every CTA computes the same decision from the same counters).
 struct SelState {
-    int k, strategy, queue_valid, done, prev_strategy, nlevels, prev_small, prefill;
+    int k, strategy, queue_valid, done, prev_strategy, nlevels, prev_small, prefill, qreset, pad_;
     long long fsize, fedges, fprev, unvisited, reached, arcs_traversed;
     long long la_cf, la_ce;    // look-ahead vertices (count, degree sum) merged into F_{k+1} before level k
     unsigned fmaxdeg;
@@ -299,9 +299,13 @@ __device__ __forceinline__ void select_step(const KArgs& a, SelState& s, bool lo
     // count pass of SS saw them, the BU / SF counters did not, and an SF queue
     // lacks them.
     const long long carry_f = s.la_cf;
+    s.qreset = 0;
     if (carry_f) {
         if (strat != XBFS_SS) { nf += carry_f; ne += s.la_ce; }
         s.queue_valid = 0;
+        // an SF step filled queue slot (k+1)%3 without the carried vertices; the
+        // queue is regenerated into that slot, whose counter must restart at 0
+        s.qreset = strat == XBFS_SF;
     }
     long long laf = 0, lae = 0;
     if (strat == XBFS_BU && st->lookahead) {
@@ -359,6 +363,7 @@ __device__ __forceinline__ void sel_load(const DevState* st, SelState& s) {
     s.arcs_traversed = __ldcg(&st->arcs_traversed);
     s.fmaxdeg = __ldcg(&st->fmaxdeg);
     s.prefill = 0;
+    s.qreset = 0;
     s.la_cf = s.la_ce = 0;   // look-ahead runs only in the persistent driver, whose state never leaves the kernel
 }
 
@@ -974,6 +979,12 @@ __device__ __forceinline__ unsigned long long globaltimer() {
     return t;
 }
 
+// 1: release-add arrival + relaxed polling with backoff + one acquire fence
+// (A/B: grid 77.2 vs 74.8 ms, s24 equal, so the SC-fence version stays default)
+#ifndef XBFS_BARRIER_V2
+#define XBFS_BARRIER_V2 0
+#endif
+
 __device__ __forceinline__ unsigned ld_acquire(const unsigned* p) {
     unsigned v;
     asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
@@ -984,20 +995,39 @@ __device__ __forceinline__ unsigned ld_acquire(const unsigned* p) {
 // run); barrier e completes when it reaches e * gridDim.x.  __syncthreads +
 // the release fence before the arrival and the acquire load after it order
 // every write of the phase before every read of the next (mutable state is
-// read through L2 everywhere).  A barrier that does not complete within 10 s
+// read through L2 everywhere).  A barrier that does not complete within 100 s
 // traps: the run fails with a CUDA error (handle poisoned) instead of hanging.
 __device__ __forceinline__ void grid_sync(unsigned* ctr, unsigned& epoch) {
     __syncthreads();
     if (threadIdx.x == 0) {
         ++epoch;
         const unsigned target = epoch * gridDim.x;
+#if XBFS_BARRIER_V2
+        // arrival with release semantics (orders this CTA's phase writes, which
+        // __syncthreads made visible to this thread, before the count); relaxed
+        // polling (no L1 invalidation per poll); one acquire fence after it
+        asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(ctr) : "memory");
+        unsigned v;
+        asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(ctr) : "memory");
+        if ((int)(v - target) < 0) {
+            const unsigned long long t0 = globaltimer();
+            int polls = 0;
+            do {
+                if (++polls > 256) __nanosleep(256);
+                if (globaltimer() - t0 > 100000000000ull) __trap();
+                asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(ctr) : "memory");
+            } while ((int)(v - target) < 0);
+        }
+        asm volatile("fence.acq_rel.gpu;" ::: "memory");
+#else
         __threadfence();
         atomicAdd(ctr, 1u);
         if ((int)(ld_acquire(ctr) - target) < 0) {
             const unsigned long long t0 = globaltimer();
             while ((int)(ld_acquire(ctr) - target) < 0)
-                if (globaltimer() - t0 > 10000000000ull) __trap();
+                if (globaltimer() - t0 > 100000000000ull) __trap();
         }
+#endif
     }
     __syncthreads();
 }
@@ -1057,6 +1087,10 @@ __global__ __launch_bounds__(kPersistThreads, kPersistBlocks) void k_persist(
         __syncthreads();
         if (LA && s.la_cf > 0) {    // look-ahead vertices of step k join F_{k+2} before step k+1
             la_merge(a, s.k);
+            grid_sync(bar, epoch);
+        }
+        if (LA && s.qreset) {       // the regenerated queue of F_{k+1} restarts its counter
+            if (blockIdx.x == 0 && threadIdx.x == 0) a.st->qctr[s.k % 3] = 0;
             grid_sync(bar, epoch);
         }
     }
