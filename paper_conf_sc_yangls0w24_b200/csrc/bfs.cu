@@ -407,20 +407,33 @@ __device__ void select_body(const KArgs& a) {
 // entry overlapping it, so tiles are balanced regardless of the degree mix
 // (hubs span many tiles, small vertices share one).  Arc a of the frontier is
 // col[a + qdelta[j]] for its owner j (binary search of qoff in shared memory).
-struct TdSmem {
-    long long off[kTile + 1];
-    long long delta[kTile + 1];
-    int v[kTile + 1];
+// TPT base tiles form one CTA step of the persistent kernel (more arcs in flight
+// per thread when its CTAs are 1024 threads wide); the per-level kernels use 1.
+// B200 A/B (1024 x 1 persistent CTAs, s24): SS 2 / SF 1 = 334 us per BFS,
+// 1/1 = 342, 2/2 = 345, 4/1 = 347 (SF's enqueue registers spill at R = 4).
+template <int TPT>
+struct TdSmemT {
+    long long off[TPT * kTile + 1];
+    long long delta[TPT * kTile + 1];
+    int v[TPT * kTile + 1];
 };
+using TdSmem = TdSmemT<1>;
+
+#ifndef XBFS_SS_TPT
+#define XBFS_SS_TPT 2
+#endif
+#ifndef XBFS_SF_TPT
+#define XBFS_SF_TPT 1
+#endif
 
 #ifndef XBFS_SF_PRECHECK_MIN
 #define XBFS_SF_PRECHECK_MIN 65536
 #endif
 constexpr long long kSfPrecheckMin = XBFS_SF_PRECHECK_MIN;   // edgesF_k above which SF probes before claiming
 
-template <int MODE, int THREADS>
+template <int MODE, int THREADS, int TPT = 1>
 __device__ __forceinline__ void td_expand_body(const KArgs& a, int k, int* __restrict__ level,
-                                               int* __restrict__ parent, TdSmem& sm, long long Fs = -1,
+                                               int* __restrict__ parent, TdSmemT<TPT>& sm, long long Fs = -1,
                                                long long Ts = -1) {
     clear_stale(a, k);
     const int in = k % 3, ob = (k + 1) % 3;
@@ -448,11 +461,12 @@ __device__ __forceinline__ void td_expand_body(const KArgs& a, int k, int* __res
     int* s_v = sm.v;
     unsigned lmax = 0;
 
-    for (long long t = blockIdx.x; t < ntiles; t += gridDim.x) {
-        const long long a0 = t * kTile;
-        const long long a1 = min(a0 + (long long)kTile, T);
-        const long long i0 = __ldcg(tfirst + t);
-        const long long i1 = (t + 1 < ntiles) ? (long long)__ldcg(tfirst + t + 1) : F - 1;
+    const long long nsteps = (ntiles + TPT - 1) / TPT;
+    for (long long t = blockIdx.x; t < nsteps; t += gridDim.x) {
+        const long long a0 = t * TPT * kTile;
+        const long long a1 = min(a0 + (long long)(TPT * kTile), T);
+        const long long i0 = __ldcg(tfirst + t * TPT);
+        const long long i1 = (t * TPT + TPT < ntiles) ? (long long)__ldcg(tfirst + t * TPT + TPT) : F - 1;
         const int nv = (int)(i1 - i0 + 1);
         __syncthreads();
         for (int i = threadIdx.x; i < nv; i += THREADS) {
@@ -463,7 +477,7 @@ __device__ __forceinline__ void td_expand_body(const KArgs& a, int k, int* __res
         __syncthreads();
         // R arcs per thread (stride THREADS: coalesced col reads), processed
         // stage by stage so the R dependent load chains are in flight together.
-        constexpr int R = kTile / THREADS;
+        constexpr int R = TPT * kTile / THREADS;
         int v[R], u[R];
         unsigned vis[R];
         bool valid[R], win[R];
@@ -1034,7 +1048,7 @@ __device__ __forceinline__ void grid_sync(unsigned* ctr, unsigned& epoch) {
 
 template <bool LA>
 union PersistSmem {
-    TdSmem td;
+    TdSmemT<(XBFS_SS_TPT > XBFS_SF_TPT ? XBFS_SS_TPT : XBFS_SF_TPT)> td;
     typename std::conditional<LA, BuSmemLa<kPersistThreads / 32>, BuSmem<kPersistThreads / 32>>::type bu;
 };
 
@@ -1074,9 +1088,11 @@ __global__ __launch_bounds__(kPersistThreads, kPersistBlocks) void k_persist(
             grid_sync(bar, epoch);
         }
         if (strat == XBFS_SF) {
-            td_expand_body<XBFS_SF, kPersistThreads>(a, k, level, parent, sm.td, s.fsize, s.fedges);
+            td_expand_body<XBFS_SF, kPersistThreads, XBFS_SF_TPT>(
+                a, k, level, parent, *reinterpret_cast<TdSmemT<XBFS_SF_TPT>*>(&sm.td), s.fsize, s.fedges);
         } else if (strat == XBFS_SS) {
-            td_expand_body<XBFS_SS, kPersistThreads>(a, k, level, parent, sm.td, s.fsize, s.fedges);
+            td_expand_body<XBFS_SS, kPersistThreads, XBFS_SS_TPT>(
+                a, k, level, parent, *reinterpret_cast<TdSmemT<XBFS_SS_TPT>*>(&sm.td), s.fsize, s.fedges);
             grid_sync(bar, epoch);
             ss_count_body(a, k);
         } else {

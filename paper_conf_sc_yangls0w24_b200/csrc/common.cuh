@@ -38,8 +38,14 @@ constexpr int kSmallBig = 8192;      // per-CTA list of higher-degree vertices (
 constexpr long long kSmallEdgesMax = 9LL * kSmallBig;  // guarantees the big list never overflows
 constexpr int kSmallMaxDeg = 512;    // frontier max degree allowed in the small mode (warp steps <= 16)
 constexpr int kLogCap = 1 << 16;     // per-level log entries kept on the device
-constexpr int kPersistThreads = 512; // persistent (one launch per BFS) driver: threads per CTA
-constexpr int kPersistBlocks = 2;    // ... CTAs per SM (64 registers per thread)
+#ifndef XBFS_PERSIST_THREADS
+#define XBFS_PERSIST_THREADS 1024
+#endif
+#ifndef XBFS_PERSIST_BLOCKS
+#define XBFS_PERSIST_BLOCKS 1
+#endif
+constexpr int kPersistThreads = XBFS_PERSIST_THREADS; // persistent (one launch per BFS) driver: threads per CTA
+constexpr int kPersistBlocks = XBFS_PERSIST_BLOCKS;   // ... CTAs per SM (64 registers per thread)
 
 struct LevelRec {
     long long fsize, fedges, unvisited, probes;
