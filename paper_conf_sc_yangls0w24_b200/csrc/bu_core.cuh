@@ -31,14 +31,14 @@ struct BuSmem {
     int list[WARPS][kBuChunkWords * 32];   // candidates of the warp's chunk
     int hard[WARPS][kBuChunkWords * 32];   // long unresolved rows (warp-cooperative)
     int hoff[WARPS][kBuChunkWords * 32];   // arcs already probed for each hard row
-    unsigned found[WARPS][kBuChunkWords];
+    unsigned found[WARPS][32];             // found words of the batch (by owning lane)
 };
 
 // ... plus the look-ahead lists (kept out of the default kernels' shared memory).
 template <int WARPS>
 struct BuSmemLa : BuSmem<WARPS> {
     int hlau[WARPS][kBuChunkWords * 32];   // F_{k+1} neighbour seen before a row went hard
-    unsigned la[WARPS][kBuChunkWords];     // look-ahead discoveries (level k+2)
+    unsigned la[WARPS][32];                // look-ahead discoveries (level k+2)
 };
 
 // Look-ahead accumulators: vertices set to level k+2 by a BU pass.
@@ -92,16 +92,42 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, Smem& sm, Publish pub
     for (long long g0 = gw; g0 < nchunks; g0 += 4 * nw) {
         const unsigned grp = grp_next;
         grp_next = load_group(g0 + 4 * nw);
-        unsigned has = __ballot_sync(FULL, grp != FULL);   // lanes whose word has a candidate
-        for (int j = 0; has; ++j, has >>= 8) {
-            if ((has & 0xffu) == 0u) continue;
+        // A sparse group (<= kCW*32 candidates over its 4 chunks, the late BU levels)
+        // runs as ONE batch: one first-probe round trip for all of it instead of one
+        // per chunk.  Dense groups run chunk by chunk.
+        const int gcnt = (int)__reduce_add_sync(FULL, (unsigned)__popc(~grp));
+        if (gcnt == 0) continue;
+        const bool whole = gcnt <= kCW * 32;
+        unsigned has = whole ? 1u : __ballot_sync(FULL, grp != FULL);   // lanes whose word has a candidate
+        for (int j = 0; has; ++j, has >>= (whole ? 1 : 8)) {
+            if (!whole && (has & 0xffu) == 0u) continue;
             const long long c = g0 + (long long)j * nw;
-            const unsigned vis_j = __shfl_sync(FULL, grp, (j << 3) | (lane & 7));
-            // 1. candidates of kCW bitmap words: ballot/popc compaction into shared memory
-            //    (the paper's count + prefix-sum + queue-write "double scan").
-            const long long w = c * kCW + lane;
-            const bool own = lane < kCW && w < b.words;
-            const unsigned vis = own ? vis_j : FULL;
+            // 1. candidates of the batch's bitmap words: ballot/popc compaction into shared
+            //    memory (the paper's count + prefix-sum + queue-write "double scan").
+            long long w;
+            bool own;
+            unsigned vis;
+            if (whole) {                 // lane l: word (l & 7) of chunk g0 + (l >> 3) * nw
+                const long long cc = g0 + (long long)(lane >> 3) * nw;
+                w = cc * kCW + (lane & 7);
+                own = cc < nchunks && w < b.words;
+                vis = own ? grp : FULL;
+            } else {                     // lanes 0..kCW-1: the words of chunk c
+                const unsigned vis_j = __shfl_sync(FULL, grp, (j << 3) | (lane & 7));
+                w = c * kCW + lane;
+                own = lane < kCW && w < b.words;
+                vis = own ? vis_j : FULL;
+            }
+            // the lane owning v's word (index into the found / look-ahead words)
+            auto slot = [&](int v) -> int {
+                const long long wv = v >> 5;
+                if (whole) {
+                    const long long cv = wv / kCW;
+                    const int jj = (cv >= g0 + nw) + (cv >= g0 + 2 * nw) + (cv >= g0 + 3 * nw);
+                    return jj * kCW + (int)(wv & (kCW - 1));
+                }
+                return (int)(wv - c * kCW);
+            };
             const unsigned cand = ~vis;
             // (chunks without a candidate were skipped above: F_{k+1} words start out
             // zero, the stale-bitmap clear of level k-1, so there is nothing to write)
@@ -115,17 +141,15 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, Smem& sm, Publish pub
             const int total = __shfl_sync(FULL, incl, 31);
             int pos = incl - cnt;
             for (unsigned bits = cand; bits; bits &= bits - 1) s_list[wib][pos++] = (int)(w * 32 + __ffs(bits) - 1);
-            if (lane < kCW) {
-                s_found[wib][lane] = 0;
-                if constexpr (LA) sm.la[wib][lane] = 0;
-            }
+            s_found[wib][lane] = 0;
+            if constexpr (LA) sm.la[wib][lane] = 0;
             __syncwarp();
             // a look-ahead discovery of v (level k+2) with parent pu (F_{k+1})
             auto la_store = [&](int v, int pu, long long deg) {
                 if constexpr (LA) {
                     b.level[v] = b.lvl + 1;
                     b.parent[v] = pu;
-                    atomicOr(&sm.la[wib][(v >> 5) - c * kCW], 1u << (v & 31));
+                    atomicOr(&sm.la[wib][slot(v)], 1u << (v & 31));
                     la.found += 1;
                     la.edges += (unsigned long long)deg;
                 }
@@ -177,7 +201,7 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, Smem& sm, Publish pub
                         if ((wd[g] >> (fu & 31)) & 1u) {
                             b.level[v] = b.lvl;
                             b.parent[v] = fu;
-                            atomicOr(&s_found[wib][(v >> 5) - c * kCW], 1u << (v & 31));
+                            atomicOr(&s_found[wib][slot(v)], 1u << (v & 31));
                             if (!H32 || (unsigned)d < dmax) {
                                 edges += (unsigned long long)d;
                                 fmax = max(fmax, (unsigned)d);
@@ -258,7 +282,7 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, Smem& sm, Publish pub
                         for (int j = 1; j < kBuBatch; ++j) if (j == hit) pu = u[j];
                         b.level[v] = b.lvl;
                         b.parent[v] = pu;
-                        atomicOr(&s_found[wib][(v >> 5) - c * kCW], 1u << (v & 31));
+                        atomicOr(&s_found[wib][slot(v)], 1u << (v & 31));
                         edges += (unsigned long long)(re - rs);
                         fmax = max(fmax, (unsigned)(re - rs));
                         ++found;
@@ -302,7 +326,7 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, Smem& sm, Publish pub
                         if (lane == first) {
                             b.level[hv] = b.lvl;
                             b.parent[hv] = u;
-                            atomicOr(&s_found[wib][(hv >> 5) - c * kCW], 1u << (hv & 31));
+                            atomicOr(&s_found[wib][slot(hv)], 1u << (hv & 31));
                             edges += (unsigned long long)(hre - hrs);
                             fmax = max(fmax, (unsigned)(hre - hrs));
                             ++found;
