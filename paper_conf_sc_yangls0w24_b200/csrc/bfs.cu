@@ -37,6 +37,11 @@ namespace xbfs {
 
 constexpr unsigned FULL = 0xffffffffu;
 
+// output fill with 256-bit stores (A/B)
+#ifndef XBFS_FILL256
+#define XBFS_FILL256 1
+#endif
+
 // BU first probe from the 4-byte head32[] (1) or the 8-byte head[] (0; A/B only)
 #ifndef XBFS_BU_H32
 #define XBFS_BU_H32 1
@@ -181,6 +186,17 @@ __device__ __forceinline__ void init_body(const KArgs& a, int* __restrict__ leve
     int4* l4 = reinterpret_cast<int4*>(level);
     int4* p4 = reinterpret_cast<int4*>(parent);
     const int4 m1 = make_int4(-1, -1, -1, -1);
+#if XBFS_FILL256
+    if ((((uintptr_t)level | (uintptr_t)parent) & 31) == 0) {
+        // one 32-byte store per sector (STG.256)
+        const long long n8 = a.n / 8;
+        for (long long i = tid; i < n8; i += nth) {
+            asm volatile("st.global.v8.b32 [%0], {%1,%1,%1,%1,%1,%1,%1,%1};" ::"l"(level + 8 * i), "r"(-1) : "memory");
+            asm volatile("st.global.v8.b32 [%0], {%1,%1,%1,%1,%1,%1,%1,%1};" ::"l"(parent + 8 * i), "r"(-1) : "memory");
+        }
+        for (long long i = n8 * 8 + tid; i < a.n; i += nth) { level[i] = -1; parent[i] = -1; }
+    } else
+#endif
     if ((((uintptr_t)level | (uintptr_t)parent) & 15) == 0) {
         for (long long i = tid; i < n4; i += nth) { l4[i] = m1; p4[i] = m1; }
         for (long long i = n4 * 4 + tid; i < a.n; i += nth) { level[i] = -1; parent[i] = -1; }

@@ -25,7 +25,10 @@ constexpr int kExpandThreads = 512;  // td_expand block
 constexpr int kBuThreads = 256;      // bu_traverse block (8 warps)
 constexpr int kBuChunkWords = 8;     // bitmap words (256 vertices) per warp chunk
 constexpr int kBuBatch = 8;          // arcs probed per lane step (one 32-byte sector of col)
-constexpr int kBuHardMin = 256;      // unresolved rows with more arcs left go warp-cooperative
+#ifndef XBFS_BU_HARD_MIN
+#define XBFS_BU_HARD_MIN 256
+#endif
+constexpr int kBuHardMin = XBFS_BU_HARD_MIN;  // unresolved rows with more arcs left go warp-cooperative
 #ifndef XBFS_BU_FIRST_ILP
 #define XBFS_BU_FIRST_ILP 4
 #endif
