@@ -156,6 +156,19 @@ xbfs_status xbfs_run(xbfs_graph* g, int64_t source, int32_t* level, int32_t* par
 xbfs_status xbfs_run_host(xbfs_graph* g, int64_t source, int32_t* level_host, int32_t* parent_host,
                           const xbfs_run_opts* opts, xbfs_run_stats* stats);
 
+/* Graph500-style multi-root run (TEPS over many roots) with HOST
+ * outputs: one BFS per sources[i], i < count, each exactly as xbfs_run.  The
+ * result of sources[i] lands in level_host/parent_host + (i % host_slots) * N
+ * (host_slots >= 1; host_slots == count keeps every result; pinned host memory
+ * gives full PCIe speed).  Pipelined: BFS i+1 runs on the handle's stream while
+ * the D2H copies of BFS i run on a second stream (two device output slots,
+ * allocated on first use, 16N bytes), so the call costs ~max(compute, copy)
+ * per root instead of their sum.  Synchronises before returning.
+ * Errors: INVALID_ARG (NULL pointer, count < 0, host_slots < 1, any source
+ * outside [0,N): checked before anything is enqueued), STATE, CUDA. */
+xbfs_status xbfs_run_host_batch(xbfs_graph* g, const int64_t* sources, int32_t count, int32_t host_slots,
+                                int32_t* level_host, int32_t* parent_host, const xbfs_run_opts* opts);
+
 /* Graph facts: N, stored arcs A, input tuples M, max degree.  Any out pointer
  * may be NULL. */
 xbfs_status xbfs_graph_info(const xbfs_graph* g, int64_t* n, int64_t* arcs, int64_t* input_edges,

@@ -113,6 +113,7 @@ void xbfs_destroy(xbfs_graph* g) {
     if (!g) return;
     cudaSetDevice(g->device);
     if (g->stream) cudaStreamSynchronize(g->stream);
+    if (g->copy_stream) cudaStreamSynchronize(g->copy_stream);
     g->drop_loops();
     void* dev[] = {g->row_ptr, g->col, g->tcount, g->nonisolated, g->visited, g->fb, g->qv,
                    g->qoff, g->qdelta, g->tile_first, g->st, g->log, g->red_scratch,
@@ -123,6 +124,11 @@ void xbfs_destroy(xbfs_graph* g) {
     if (g->ev0) cudaEventDestroy(g->ev0);
     if (g->ev1) cudaEventDestroy(g->ev1);
     for (cudaEvent_t e : g->prof_events) cudaEventDestroy(e);
+    for (int s = 0; s < 2; ++s) {
+        if (g->ev_done[s]) cudaEventDestroy(g->ev_done[s]);
+        if (g->ev_copied[s]) cudaEventDestroy(g->ev_copied[s]);
+    }
+    if (g->copy_stream) cudaStreamDestroy(g->copy_stream);
     cudaGetLastError();
     delete g;
 }

@@ -1511,16 +1511,63 @@ extern "C" xbfs_status xbfs_run(xbfs_graph* g, int64_t source, int32_t* level, i
     return run_impl(g, source, level, parent, opts, stats);
 }
 
+// Two device output slots + a copy stream for the host-output calls (lazily, 16N bytes).
+static xbfs_status ensure_host_scratch(xbfs_graph* g) {
+    if (!g->scratch_level) {
+        XBFS_CUDA(g, cudaMalloc(&g->scratch_level, 2 * g->n * sizeof(int)));
+        XBFS_CUDA(g, cudaMalloc(&g->scratch_parent, 2 * g->n * sizeof(int)));
+    }
+    if (!g->copy_stream) {
+        XBFS_CUDA(g, cudaStreamCreateWithFlags(&g->copy_stream, cudaStreamNonBlocking));
+        for (int s = 0; s < 2; ++s) {
+            XBFS_CUDA(g, cudaEventCreateWithFlags(&g->ev_done[s], cudaEventDisableTiming));
+            XBFS_CUDA(g, cudaEventCreateWithFlags(&g->ev_copied[s], cudaEventDisableTiming));
+        }
+    }
+    return XBFS_OK;
+}
+
+extern "C" xbfs_status xbfs_run_host_batch(xbfs_graph* g, const int64_t* sources, int32_t count, int32_t host_slots,
+                                           int32_t* level_host, int32_t* parent_host, const xbfs_run_opts* opts) {
+    if (!g) return set_error(XBFS_ERR_INVALID_ARG, "xbfs_run_host_batch: NULL handle");
+    if (count < 0 || host_slots < 1) return set_error(XBFS_ERR_INVALID_ARG, "xbfs_run_host_batch: count < 0 or host_slots < 1");
+    if (count == 0) return XBFS_OK;
+    if (!sources || !level_host || !parent_host)
+        return set_error(XBFS_ERR_INVALID_ARG, "xbfs_run_host_batch: NULL sources/level/parent");
+    for (int32_t i = 0; i < count; ++i)
+        if (sources[i] < 0 || sources[i] >= g->n)
+            return set_error(XBFS_ERR_INVALID_ARG, "xbfs_run_host_batch: sources[%d] = %lld outside [0, %lld)", i,
+                             (long long)sources[i], g->n);
+    if (g->poisoned) return set_error(XBFS_ERR_STATE, "handle poisoned by an earlier failure");
+    XBFS_CUDA(g, cudaSetDevice(g->device));
+    XBFS_TRY(ensure_host_scratch(g));
+    const size_t bytes = (size_t)g->n * sizeof(int);
+    for (int32_t i = 0; i < count; ++i) {
+        const int s = i & 1;
+        int* lv = g->scratch_level + (size_t)s * g->n;
+        int* pa = g->scratch_parent + (size_t)s * g->n;
+        // slot s is free once the D2H copies of BFS i-2 have drained
+        if (i >= 2) XBFS_CUDA(g, cudaStreamWaitEvent(g->stream, g->ev_copied[s], 0));
+        XBFS_TRY(run_impl(g, sources[i], lv, pa, opts, nullptr));
+        XBFS_CUDA(g, cudaEventRecord(g->ev_done[s], g->stream));
+        XBFS_CUDA(g, cudaStreamWaitEvent(g->copy_stream, g->ev_done[s], 0));
+        const size_t off = (size_t)(i % host_slots) * g->n;
+        XBFS_CUDA(g, cudaMemcpyAsync(level_host + off, lv, bytes, cudaMemcpyDeviceToHost, g->copy_stream));
+        XBFS_CUDA(g, cudaMemcpyAsync(parent_host + off, pa, bytes, cudaMemcpyDeviceToHost, g->copy_stream));
+        XBFS_CUDA(g, cudaEventRecord(g->ev_copied[s], g->copy_stream));
+    }
+    XBFS_CUDA(g, cudaStreamSynchronize(g->copy_stream));
+    XBFS_CUDA(g, cudaStreamSynchronize(g->stream));
+    return XBFS_OK;
+}
+
 extern "C" xbfs_status xbfs_run_host(xbfs_graph* g, int64_t source, int32_t* level_host, int32_t* parent_host,
                                      const xbfs_run_opts* opts, xbfs_run_stats* stats) {
     if (!g) return set_error(XBFS_ERR_INVALID_ARG, "xbfs_run_host: NULL handle");
     if (!level_host || !parent_host) return set_error(XBFS_ERR_INVALID_ARG, "xbfs_run_host: NULL level/parent");
     if (g->poisoned) return set_error(XBFS_ERR_STATE, "handle poisoned by an earlier failure");
     XBFS_CUDA(g, cudaSetDevice(g->device));
-    if (!g->scratch_level) {
-        XBFS_CUDA(g, cudaMalloc(&g->scratch_level, g->n * sizeof(int)));
-        XBFS_CUDA(g, cudaMalloc(&g->scratch_parent, g->n * sizeof(int)));
-    }
+    XBFS_TRY(ensure_host_scratch(g));
     xbfs_status s = run_impl(g, source, g->scratch_level, g->scratch_parent, opts, stats);
     if (s != XBFS_OK) return s;
     XBFS_CUDA(g, cudaMemcpyAsync(level_host, g->scratch_level, g->n * sizeof(int), cudaMemcpyDeviceToHost, g->stream));

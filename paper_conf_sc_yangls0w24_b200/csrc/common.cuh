@@ -157,8 +157,10 @@ struct xbfs_graph {
     xbfs::HostCtl* hctl = nullptr;       // pinned host
     xbfs::HostCtl* hctl_dev = nullptr;   // its device alias
     unsigned long long* red_scratch = nullptr;  // reductions for stats
-    int* scratch_level = nullptr;        // xbfs_run_host device scratch
+    int* scratch_level = nullptr;        // xbfs_run_host device scratch: 2 slots of N (batch pipelining)
     int* scratch_parent = nullptr;
+    cudaStream_t copy_stream = nullptr;  // D2H of xbfs_run_host_batch
+    cudaEvent_t ev_done[2] = {nullptr, nullptr}, ev_copied[2] = {nullptr, nullptr};
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
     int dbits = 40;
     // CUDA-graph device loop (built lazily)

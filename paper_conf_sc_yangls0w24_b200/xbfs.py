@@ -75,6 +75,7 @@ def _load():
     L.xbfs_reorder.argtypes = [P, i32]
     L.xbfs_run.argtypes = [P, i64, P, P, ctypes.POINTER(RunOpts), ctypes.POINTER(RunStats)]
     L.xbfs_run_host.argtypes = [P, i64, P, P, ctypes.POINTER(RunOpts), ctypes.POINTER(RunStats)]
+    L.xbfs_run_host_batch.argtypes = [P, P, i32, i32, P, P, ctypes.POINTER(RunOpts)]
     L.xbfs_graph_info.argtypes = [P, P, P, P, P]
     L.xbfs_copy_csr.argtypes = [P, P, P]
     L.xbfs_destroy.argtypes = [P]
@@ -83,7 +84,8 @@ def _load():
     L.xbfs_run_opts_default.argtypes = [ctypes.POINTER(RunOpts)]
     L.xbfs_run_opts_default.restype = None
     L.xbfs_compiled_arch.restype = i32
-    for fn in ("xbfs_build_csr", "xbfs_reorder", "xbfs_run", "xbfs_run_host", "xbfs_graph_info", "xbfs_copy_csr"):
+    for fn in ("xbfs_build_csr", "xbfs_reorder", "xbfs_run", "xbfs_run_host", "xbfs_run_host_batch",
+               "xbfs_graph_info", "xbfs_copy_csr"):
         getattr(L, fn).restype = ctypes.c_int
     if L.xbfs_compiled_arch() != 100:
         raise ImportError("libxbfs.so was not built for sm_100a")
@@ -94,6 +96,7 @@ lib = _load()
 
 #: every symbol include/xbfs.h declares (checked by tests/test_abi.py)
 EXPORTS = ("xbfs_run_opts_default", "xbfs_build_csr", "xbfs_reorder", "xbfs_run", "xbfs_run_host",
+           "xbfs_run_host_batch",
            "xbfs_graph_info", "xbfs_copy_csr", "xbfs_destroy", "xbfs_last_error", "xbfs_compiled_arch")
 
 
@@ -136,6 +139,17 @@ def xbfs_run(g: int, source: int, level, parent, opts: RunOpts | None = None, st
 def xbfs_run_host(g: int, source: int, level, parent, opts: RunOpts | None = None, stats: RunStats | None = None):
     _check(lib.xbfs_run_host(g, source, _ptr(level), _ptr(parent), ctypes.byref(opts) if opts else None,
                              ctypes.byref(stats) if stats else None))
+
+
+def xbfs_run_host_batch(g: int, sources, level, parent, host_slots: int | None = None,
+                        opts: RunOpts | None = None):
+    """sources: int64 array of K roots; level/parent: host int32 arrays of host_slots * N
+    (host_slots defaults to K); root i's result lands in slot i % host_slots."""
+    src = np.ascontiguousarray(np.asarray(sources, dtype=np.int64))
+    k = int(src.size)
+    slots = k if host_slots is None else int(host_slots)
+    _check(lib.xbfs_run_host_batch(g, src.ctypes.data if k else None, k, max(slots, 1) if k == 0 else slots,
+                                   _ptr(level), _ptr(parent), ctypes.byref(opts) if opts else None))
 
 
 def xbfs_graph_info(g: int):
@@ -288,6 +302,11 @@ class Graph:
         sb = _StatsBuf() if stats else None
         xbfs_run_host(self._h, int(source), level_host, parent_host, make_run_opts(**opts), sb.c if sb else None)
         return sb.result() if sb else None
+
+    def run_host_batch(self, sources, level_host, parent_host, host_slots: int | None = None, **opts):
+        """Pipelined multi-root BFS into host arrays (xbfs_run_host_batch): D2H of root i
+        overlaps the BFS of root i+1."""
+        xbfs_run_host_batch(self._h, sources, level_host, parent_host, host_slots, make_run_opts(**opts))
 
     def csr(self):
         return xbfs_copy_csr(self._h)

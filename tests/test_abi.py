@@ -52,6 +52,7 @@ def test_invalid_arguments_do_not_touch_cuda(xb):
     assert xb.lib.xbfs_build_csr(None, None, 0, 1 << 31, None, ctypes.byref(h)) == xb.XBFS_ERR_INVALID_ARG
     assert xb.lib.xbfs_run(None, 0, None, None, None, None) == xb.XBFS_ERR_INVALID_ARG
     assert xb.lib.xbfs_reorder(None, 1) == xb.XBFS_ERR_INVALID_ARG
+    assert xb.lib.xbfs_run_host_batch(None, None, 1, 1, None, None, None) == xb.XBFS_ERR_INVALID_ARG
     assert xb.lib.xbfs_graph_info(None, None, None, None, None) == xb.XBFS_ERR_INVALID_ARG
     xb.lib.xbfs_destroy(None)  # NULL-safe
     from paper_conf_sc_yangls0w24_b200 import dist
