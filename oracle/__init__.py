@@ -8,8 +8,8 @@ header and DESIGN.md §3); pins live in ``tests/test_oracle.py``.
 
 Parity status per function:
   build_csr, reorder, bfs, validate, input_edges, level_stats, select,
-  byte_replay — all pinned (closed forms, scipy brute force, mutation tests,
-  hand-computed replay).  The paper's own worked example (Figs 1-4) is lost:
+  byte_replay, build_csr_directed, validate_directed — all pinned (closed
+  forms, scipy brute force, mutation tests, hand-computed replay).  The paper's own worked example (Figs 1-4) is lost:
   "parity unpinned" for that example only.
 """
 from __future__ import annotations
@@ -62,6 +62,10 @@ def lib():
         L.oracle_byte_replay.restype = i64
         L.oracle_bu_probes.argtypes = [i64, P, P, P, i32]
         L.oracle_bu_probes.restype = i64
+        L.oracle_build_csr_directed.argtypes = [i64, i64, P, P, P, P, P]
+        L.oracle_build_csr_directed.restype = ctypes.c_int
+        L.oracle_validate_directed.argtypes = [i64, P, P, i64, P, P, i64, P, P]
+        L.oracle_validate_directed.restype = ctypes.c_int
         _lib = L
     return _lib
 
@@ -98,6 +102,28 @@ def build_csr(n: int, src, dst) -> CSR:
     if rc != 0:
         raise ValueError(f"oracle_build_csr failed rc={rc}")
     return CSR(n, row_ptr, col[: arcs.value].copy())
+
+
+def build_csr_directed(n: int, src, dst) -> CSR:
+    """f4 / reading R-9: out-arc CSR of the tuples taken as arcs src -> dst."""
+    src, dst = _u32(src), _u32(dst)
+    m = src.shape[0]
+    row_ptr = np.zeros(n + 1, dtype=np.int64)
+    col = np.zeros(max(m, 1), dtype=np.int32)
+    arcs = ctypes.c_int64(0)
+    rc = lib().oracle_build_csr_directed(n, m, _p(src), _p(dst), _p(row_ptr), _p(col), ctypes.byref(arcs))
+    if rc != 0:
+        raise ValueError(f"oracle_build_csr_directed failed rc={rc}")
+    return CSR(n, row_ptr, col[: arcs.value].copy())
+
+
+def validate_directed(g: CSR, src, dst, source: int, level, parent) -> int:
+    """Graph500 checks restated for arcs (oracle.c); g = build_csr_directed's CSR."""
+    src, dst = _u32(src), _u32(dst)
+    level = np.ascontiguousarray(level, dtype=np.int32)
+    parent = np.ascontiguousarray(parent, dtype=np.int32)
+    return lib().oracle_validate_directed(g.n, _p(g.row_ptr), _p(g.col), src.shape[0], _p(src), _p(dst),
+                                          int(source), _p(level), _p(parent))
 
 
 def reorder(g: CSR) -> CSR:

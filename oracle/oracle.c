@@ -28,6 +28,15 @@
  *                      (rule unstated in the paper: reading C-10).
  *   oracle_byte_replay O-8: algorithmic bytes of one BFS given the per-level
  *                      strategy sequence.
+ *   oracle_build_csr_directed  f4 (directed graphs; reading
+ *                      R-9): out-arc CSR of the tuples taken as arcs i -> j,
+ *                      self-loops and duplicate arcs dropped, rows id-sorted.
+ *                      oracle_bfs / oracle_level_stats / oracle_reorder apply
+ *                      unchanged to it (BFS follows out-arcs).
+ *   oracle_validate_directed  the Graph500 checks restated for arcs: V1, V2,
+ *                      V3 as undirected; V4 the tree arc parent[v] -> v exists;
+ *                      V5 for every tuple (i,j), i != j: i reached implies j
+ *                      reached with level[j] <= level[i] + 1.
  *
  * Parity pins: tests/test_oracle.py (closed forms, scipy brute force,
  * validator mutation tests, hand-computed byte replay).
@@ -289,4 +298,79 @@ int64_t oracle_bu_probes(int64_t n, const int64_t* row_ptr, const int32_t* col,
         probes += pr;
     }
     return probes;
+}
+
+/* ------------------------------------------- f4: directed graphs (R-9) */
+
+/* Out-arc CSR: every tuple (i,j), i != j, is the arc i -> j.  Same two-pass
+ * counting sort as oracle_build_csr, one arc per tuple: pass 1 groups arcs by
+ * target j, pass 2 walks targets j = 0..n-1 and appends j to the row of each
+ * source i, so every row receives its targets in ascending id order;
+ * duplicates are then adjacent and dropped.  col capacity >= m. */
+int oracle_build_csr_directed(int64_t n, int64_t m, const uint32_t* src, const uint32_t* dst,
+                              int64_t* row_ptr, int32_t* col, int64_t* arcs_out) {
+    if (n <= 0 || m < 0 || !row_ptr || !col || !arcs_out) return 1;
+    for (int64_t e = 0; e < m; ++e)
+        if (src[e] >= (uint64_t)n || dst[e] >= (uint64_t)n) return 1;
+    int64_t* tstart = (int64_t*)calloc((size_t)n + 1, sizeof(int64_t));   /* by target */
+    int64_t* start = (int64_t*)calloc((size_t)n + 1, sizeof(int64_t));    /* by source */
+    int64_t* cur = (int64_t*)malloc(((size_t)n + 1) * sizeof(int64_t));
+    int32_t* tmp = (int32_t*)malloc((size_t)(m > 0 ? m : 1) * sizeof(int32_t));
+    if (!tstart || !start || !cur || !tmp) { free(tstart); free(start); free(cur); free(tmp); return 2; }
+    for (int64_t e = 0; e < m; ++e) {
+        if (src[e] == dst[e]) continue;              /* self-loop dropped */
+        tstart[dst[e] + 1]++;
+        start[src[e] + 1]++;
+    }
+    for (int64_t v = 0; v < n; ++v) { tstart[v + 1] += tstart[v]; start[v + 1] += start[v]; }
+    /* pass 1: sources grouped by target */
+    memcpy(cur, tstart, (size_t)n * sizeof(int64_t));
+    for (int64_t e = 0; e < m; ++e) {
+        if (src[e] == dst[e]) continue;
+        tmp[cur[dst[e]]++] = (int32_t)src[e];
+    }
+    /* pass 2: row i receives j for every arc i -> j, j ascending */
+    memcpy(cur, start, (size_t)n * sizeof(int64_t));
+    for (int64_t j = 0; j < n; ++j)
+        for (int64_t p = tstart[j]; p < tstart[j + 1]; ++p)
+            col[cur[tmp[p]]++] = (int32_t)j;
+    int64_t out = 0;
+    for (int64_t v = 0; v < n; ++v) {
+        int64_t b = start[v], e = start[v + 1];
+        row_ptr[v] = out;
+        for (int64_t i = b; i < e; ++i) {
+            if (i > b && col[i] == col[i - 1]) continue;
+            col[out++] = col[i];
+        }
+    }
+    row_ptr[n] = out;
+    *arcs_out = out;
+    free(tstart); free(start); free(cur); free(tmp);
+    return 0;
+}
+
+/* Validation of a BFS over arcs.  row_ptr/col: oracle_build_csr_directed's
+ * id-sorted out-arc CSR.  Same bitmask as oracle_validate. */
+int oracle_validate_directed(int64_t n, const int64_t* row_ptr, const int32_t* col,
+                             int64_t m, const uint32_t* src, const uint32_t* dst, int64_t s,
+                             const int32_t* level, const int32_t* parent) {
+    int bad = 0;
+    if (s < 0 || s >= n) return V_RANGE;
+    if (parent[s] != s || level[s] != 0) bad |= V1_ROOT;                      /* V1 */
+    for (int64_t v = 0; v < n; ++v) {
+        int reached_l = level[v] >= 0, reached_p = parent[v] >= 0;
+        if (reached_l != reached_p) { bad |= V2_REACH_CONSISTENT; continue; } /* V2 */
+        if (parent[v] >= n || level[v] < -1) { bad |= V_RANGE; continue; }
+        if (!reached_l || v == s) continue;
+        int32_t p = parent[v];
+        if (level[p] != level[v] - 1) bad |= V3_LEVEL_STEP;                   /* V3 */
+        if (!has_arc(row_ptr, col, p, (int32_t)v)) bad |= V4_TREE_EDGE;       /* V4: arc p -> v */
+    }
+    for (int64_t e = 0; e < m; ++e) {                                          /* V5 */
+        if (src[e] == dst[e]) continue;
+        int32_t li = level[src[e]], lj = level[dst[e]];
+        if (li < 0) continue;                        /* nothing follows from an unreached tail */
+        if (lj < 0 || lj > li + 1) bad |= V5_EDGE_SPAN;
+    }
+    return bad;
 }

@@ -381,3 +381,103 @@ def test_bu_probes_hand_computed():
     # k=0 (F_0 = {1}): v0 row [4,1,2,3] hits 1 at index 1 -> 2; v2, v3 -> 1 each (deg);
     # v4 -> 2; v5 -> 2; v6 -> 1
     assert oracle.bu_probes(g, level, 0) == 2 + 1 + 1 + 2 + 2 + 1
+
+
+# ------------------------------------------------- f4: directed graphs (R-9)
+
+def test_directed_path_one_way():
+    """0 -> 1 -> 2 -> 3: levels from 0 are 0..3; from 3 nothing else is reachable
+    (the undirected build would reach all four)."""
+    n, src, dst = _graph(4, [(0, 1), (1, 2), (2, 3)])
+    g = oracle.build_csr_directed(n, src, dst)
+    assert g.row_ptr.tolist() == [0, 1, 2, 3, 3] and g.col.tolist() == [1, 2, 3]
+    lv, pa, nl = oracle.bfs(g, 0)
+    assert lv.tolist() == [0, 1, 2, 3] and pa.tolist() == [0, 0, 1, 2] and nl == 4
+    lv, pa, nl = oracle.bfs(g, 3)
+    assert lv.tolist() == [-1, -1, -1, 0] and nl == 1
+    assert oracle.validate_directed(g, src, dst, 3, lv, pa) == 0
+
+
+def test_directed_cycle_closed_form():
+    """Directed n-cycle i -> i+1 (mod n): level(v) = (v - s) mod n."""
+    n = 37
+    e = [(i, (i + 1) % n) for i in range(n)]
+    n, src, dst = _graph(n, e)
+    g = oracle.build_csr_directed(n, src, dst)
+    for s in (0, 5, 36):
+        lv, pa, nl = oracle.bfs(g, s)
+        assert lv.tolist() == [(v - s) % n for v in range(n)] and nl == n
+        assert oracle.validate_directed(g, src, dst, s, lv, pa) == 0
+
+
+@pytest.mark.parametrize("seed", range(8))
+def test_directed_bfs_matches_scipy(seed):
+    rng = np.random.default_rng(500 + seed)
+    n = int(rng.integers(2, 64))
+    e = _random_graph(rng, n, int(rng.integers(0, 4 * n)))
+    n, src, dst = _graph(n, e)
+    g = oracle.build_csr_directed(n, src, dst)
+    mask = src != dst
+    A = sp.coo_matrix((np.ones(mask.sum()), (src[mask], dst[mask])), shape=(n, n)).tocsr()
+    D = shortest_path(A, directed=True, unweighted=True)
+    for s in range(n):
+        level, parent, _ = oracle.bfs(g, s)
+        expect = np.where(np.isinf(D[s]), -1, D[s]).astype(np.int64)
+        assert np.array_equal(level, expect)
+        assert oracle.validate_directed(g, src, dst, s, level, parent) == 0
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_directed_csr_matches_set_build(seed):
+    rng = np.random.default_rng(600 + seed)
+    n = int(rng.integers(1, 1 << 11))
+    e = _random_graph(rng, n, int(rng.integers(0, 8 * n)))
+    n, src, dst = _graph(n, e)
+    g = oracle.build_csr_directed(n, src, dst)
+    rows = [set() for _ in range(n)]
+    for u, v in zip(src.tolist(), dst.tolist()):
+        if u != v:
+            rows[u].add(v)
+    rp = np.concatenate([[0], np.cumsum([len(r) for r in rows])])
+    col = np.array([c for r in rows for c in sorted(r)], dtype=np.int32)
+    assert np.array_equal(g.row_ptr, rp)
+    assert np.array_equal(g.col, col)
+
+
+def test_directed_validator_rejects_mutations():
+    rng = np.random.default_rng(21)
+    n = 300
+    n, src, dst = _graph(n, rng.integers(0, n, (1500, 2)))
+    g = oracle.build_csr_directed(n, src, dst)
+    s = int(src[0])
+    level, parent, _ = oracle.bfs(g, s)
+    assert oracle.validate_directed(g, src, dst, s, level, parent) == 0
+    # a tree arc used backwards: v's parent replaced by a vertex one level up that v
+    # only has an IN-arc from... pick u at level(v)-1 with arc v -> u but not u -> v
+    out = lambda u: set(g.col[g.row_ptr[u]:g.row_ptr[u + 1]].tolist())
+    done = False
+    for v in np.flatnonzero(level >= 2):
+        for u in np.flatnonzero(level == level[v] - 1):
+            if u in out(v) and v not in out(u):
+                p = parent.copy(); p[v] = int(u)
+                assert oracle.validate_directed(g, src, dst, s, level, p) & oracle.V4_TREE_EDGE
+                done = True
+                break
+        if done:
+            break
+    assert done
+    # an arc i -> j skipping levels: pretend j is two levels deeper than allowed
+    i = int(np.flatnonzero(level == 1)[0])
+    j = next(iter(out(i)))
+    lv = level.copy(); lv[j] = level[i] + 2
+    assert oracle.validate_directed(g, src, dst, s, lv, parent) != 0
+    # unreached head of a reached tail
+    lv = level.copy(); p = parent.copy(); lv[j] = -1; p[j] = -1
+    if j != s:
+        assert oracle.validate_directed(g, src, dst, s, lv, p) & oracle.V5_EDGE_SPAN
+    # the undirected validator would reject a valid directed tree of a one-way path
+    n2, s2, d2 = _graph(3, [(0, 1), (1, 2)])
+    g2 = oracle.build_csr_directed(n2, s2, d2)
+    lv2, pa2, _ = oracle.bfs(g2, 1)
+    assert oracle.validate_directed(g2, s2, d2, 1, lv2, pa2) == 0
+    assert oracle.validate(oracle.build_csr(n2, s2, d2), s2, d2, 1, lv2, pa2) & oracle.V5_EDGE_SPAN
