@@ -56,6 +56,10 @@ typedef struct {
     void* stream;            /* cudaStream_t for all work of this handle; NULL = legacy default */
     int32_t edges_on_device; /* 1: src/dst are device pointers; 0: host pointers */
     int32_t keep_duplicates; /* 0 (default): drop duplicate arcs (reading C-3) */
+    int32_t directed;        /* 1: tuple (i,j) is the arc i -> j only (reading R-9): top-down
+                                steps follow out-arcs, bottom-up steps search in-arcs (a second, transposed
+                                CSR), BU candidates are vertices with in-degree > 0.  Runs on the persistent
+                                driver only (driver 0/3, no look-ahead); 0 (default): symmetric graph */
 } xbfs_build_opts;
 
 /* Options for xbfs_run.  xbfs_run_opts_default() fills the paper's values. */

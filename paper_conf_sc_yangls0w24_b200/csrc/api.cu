@@ -56,6 +56,10 @@ xbfs::KArgs xbfs_graph::kargs() const {
     a.arcs = arcs;
     a.dbits = dbits;
     a.track_max = 1;
+    a.directed = directed;
+    a.bu_row_ptr = directed ? in_row_ptr : row_ptr;
+    a.bu_col = directed ? in_col : col;
+    a.bu_head32 = directed ? in_head32 : head32;
     return a;
 }
 
@@ -117,7 +121,8 @@ void xbfs_destroy(xbfs_graph* g) {
     g->drop_loops();
     void* dev[] = {g->row_ptr, g->col, g->tcount, g->nonisolated, g->visited, g->fb, g->qv,
                    g->qoff, g->qdelta, g->tile_first, g->st, g->log, g->red_scratch,
-                   g->scratch_level, g->scratch_parent, g->head, g->head32};
+                   g->scratch_level, g->scratch_parent, g->head, g->head32,
+                   g->in_row_ptr, g->in_col, g->in_head32};
     for (void* p : dev)
         if (p) cudaFree(p);
     if (g->hctl) cudaFreeHost(g->hctl);

@@ -239,7 +239,9 @@ __device__ __forceinline__ void seed_body(const KArgs& a, int* level, int* paren
     const long long rs = a.row_ptr[s], deg = a.row_ptr[s + 1] - rs;
     level[s] = 0;
     parent[s] = (int)s;
-    atomicOr(a.visited + (s >> 5), 1u << (s & 31));
+    // the source was a BU candidate (counted in U_0) iff init left its visited bit clear
+    const unsigned sbit = 1u << (s & 31);
+    const bool s_cand = !(atomicOr(a.visited + (s >> 5), sbit) & sbit);
     atomicOr(a.fb[0] + (s >> 5), 1u << (s & 31));
     a.qv[0][0] = (int)s;
     a.qoff[0][0] = 0;
@@ -262,7 +264,7 @@ __device__ __forceinline__ void seed_body(const KArgs& a, int* level, int* paren
     st->fsize = 1;
     st->fedges = deg;
     st->fprev = 0;
-    st->unvisited = nonisolated_count - (deg > 0 ? 1 : 0);
+    st->unvisited = nonisolated_count - (s_cand ? 1 : 0);
     for (int i = 0; i < 3; ++i) {
         st->acc_found[i] = st->acc_edges[i] = st->acc_probes[i] = 0;
         st->acc_la_found[i] = st->acc_la_edges[i] = 0;
@@ -713,10 +715,10 @@ __device__ __forceinline__ void bu_body(const KArgs& a, const int* kp, int* __re
     b.visited = a.visited;
     b.words = a.words;
     b.head = a.head;
-    b.head32 = a.head32;
+    b.head32 = a.bu_head32;          // in-arc CSR on a directed graph (f4, R-9)
     b.idbits = a.idbits;
-    b.row_ptr = a.row_ptr;
-    b.col = a.col;
+    b.row_ptr = a.bu_row_ptr;
+    b.col = a.bu_col;
     b.level = level;
     b.parent = parent;
     b.lvl = lvl;
@@ -740,6 +742,10 @@ __device__ __forceinline__ void bu_body(const KArgs& a, const int* kp, int* __re
         }
     }
     k = *(const volatile int*)kp;
+    // directed graph: the BU rows are in-arc rows, whose lengths are not the out-degrees
+    // edgesF_{k+1} needs; the count pass (ss_count_body) that follows supplies |F_{k+1}|
+    // and edgesF_{k+1} from the out-arc head[] instead
+    if (a.directed) found = edges = 0;
     if (lane == 0 && (found | edges | probes)) {
         atomicAdd(&a.st->acc_found[k % 3], found);
         atomicAdd(&a.st->acc_edges[k % 3], edges);
@@ -1113,6 +1119,10 @@ __global__ __launch_bounds__(kPersistThreads, kPersistBlocks) void k_persist(
             ss_count_body(a, k);
         } else {
             bu_body<kPersistThreads / 32, LA>(a, &s.k, level, parent, sm.bu, s.prefill);
+            if (a.directed) {       // |F_{k+1}|, edgesF_{k+1} over out-arcs (see bu_body)
+                grid_sync(bar, epoch);
+                ss_count_body(a, k);
+            }
         }
         grid_sync(bar, epoch);
         if (threadIdx.x == 0) select_step(a, s, blockIdx.x == 0, blockIdx.x == 0 ? globaltimer() : 0ull);
@@ -1423,6 +1433,10 @@ static xbfs_status run_impl(xbfs_graph* g, int64_t source, int32_t* level, int32
     const bool host_only = (stats && stats->kernel_capacity > 0) || (o.plan && o.plan_len > 0);
     const bool use_persist = (o.driver == 0 || o.driver == 3) && !host_only;
     const bool use_graph = o.driver == 2 && !host_only;
+    if (g->directed && (!use_persist || o.lookahead))
+        return set_error(XBFS_ERR_UNSUPPORTED,
+                         "directed graphs run on the persistent driver only (driver 0/3, no plan, no per-launch "
+                         "profiling, no look-ahead)");
     if (o.lookahead && !use_persist)
         return set_error(XBFS_ERR_INVALID_ARG, "lookahead needs the persistent driver (driver 0/3, no plan/profiling)");
     // selection parameters live in the device state

@@ -28,7 +28,8 @@ template <typename IdT>
 __global__ __launch_bounds__(kB) void k_check_and_pack(const IdT* __restrict__ src, const IdT* __restrict__ dst,
                                                        long long m, long long n, int nb,
                                                        unsigned long long* __restrict__ keys,
-                                                       int* __restrict__ tcount, int* __restrict__ bad) {
+                                                       int* __restrict__ tcount, int* __restrict__ bad,
+                                                       int directed) {
     const unsigned long long sentinel = (nb >= 32) ? ~0ull : ((1ull << (2 * nb)) - 1ull);
     for (long long e = blockIdx.x * (long long)blockDim.x + threadIdx.x; e < m;
          e += (long long)gridDim.x * blockDim.x) {
@@ -43,7 +44,8 @@ __global__ __launch_bounds__(kB) void k_check_and_pack(const IdT* __restrict__ s
             keys[2 * e] = keys[2 * e + 1] = sentinel;
         } else {                   // both arcs of the undirected edge (reading C-2)
             keys[2 * e] = ((unsigned long long)u << nb) | (unsigned long long)v;
-            keys[2 * e + 1] = ((unsigned long long)v << nb) | (unsigned long long)u;
+            keys[2 * e + 1] = directed ? sentinel   // arc u -> v only (f4, reading R-9)
+                                       : ((unsigned long long)v << nb) | (unsigned long long)u;
         }
     }
 }
@@ -111,7 +113,7 @@ __global__ __launch_bounds__(kB) void k_head(const long long* __restrict__ row_p
     for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < n;
          v += (long long)gridDim.x * blockDim.x) {
         const long long rs = row_ptr[v], d = row_ptr[v + 1] - rs;
-        head[v] = ((unsigned long long)d << 32) | (d > 0 ? (unsigned)col[rs] : 0xffffffffu);
+        if (head) head[v] = ((unsigned long long)d << 32) | (d > 0 ? (unsigned)col[rs] : 0xffffffffu);
         const unsigned dc = d < (long long)dmax ? (unsigned)d : dmax;
         head32[v] = (idbits >= 32 ? 0u : (dc << idbits)) | (d > 0 ? (unsigned)col[rs] : 0u);
     }
@@ -120,10 +122,12 @@ __global__ __launch_bounds__(kB) void k_head(const long long* __restrict__ row_p
 // Reorder keys: (row << db) | (maxdeg - deg(col))  -> degree descending within the
 // row; the radix sort is stable so ties keep ascending id order (reading C-12).
 // mode 0 keys: (row << nb) | col  -> id order.
+// deg_rp: the row_ptr degrees are read from (the out-arc CSR also for the in-arc one).
 __global__ __launch_bounds__(kB) void k_reorder_keys(const long long* __restrict__ row_ptr,
                                                      const int* __restrict__ col, long long n, long long a,
                                                      int mode, int shift, unsigned long long maxdeg,
-                                                     unsigned long long* __restrict__ keys) {
+                                                     unsigned long long* __restrict__ keys,
+                                                     const long long* __restrict__ deg_rp) {
     for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < a;
          i += (long long)gridDim.x * blockDim.x) {
         // row of arc i: last r with row_ptr[r] <= i
@@ -133,9 +137,25 @@ __global__ __launch_bounds__(kB) void k_reorder_keys(const long long* __restrict
             if (row_ptr[mid] <= i) lo = mid; else hi = mid - 1;
         }
         int c = col[i];
-        unsigned long long low = mode == 1 ? maxdeg - (unsigned long long)(row_ptr[c + 1] - row_ptr[c])
+        unsigned long long low = mode == 1 ? maxdeg - (unsigned long long)(deg_rp[c + 1] - deg_rp[c])
                                            : (unsigned long long)c;
         keys[i] = ((unsigned long long)lo << shift) | low;
+    }
+}
+
+// Directed graphs (f4): key (col << nb) | row of every out-arc, i.e. the arc as a row of
+// the transposed (in-arc) CSR; sorted and split like the input tuples.
+__global__ __launch_bounds__(kB) void k_transpose_keys(const long long* __restrict__ row_ptr,
+                                                       const int* __restrict__ col, long long n, long long a,
+                                                       int nb, unsigned long long* __restrict__ keys) {
+    for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < a;
+         i += (long long)gridDim.x * blockDim.x) {
+        long long lo = 0, hi = n - 1;
+        while (lo < hi) {
+            long long mid = (lo + hi + 1) >> 1;
+            if (row_ptr[mid] <= i) lo = mid; else hi = mid - 1;
+        }
+        keys[i] = ((unsigned long long)col[i] << nb) | (unsigned long long)lo;
     }
 }
 
@@ -162,7 +182,7 @@ xbfs_status pack_edges(xbfs_graph* g, const void* src, const void* dst, long lon
             pd = dd;
         }
         k_check_and_pack<IdT><<<grid_for(c), kB, 0, g->stream>>>(ps, pd, c, g->n, nb, keys + 2 * e0,
-                                                                 g->tcount, bad);
+                                                                 g->tcount, bad, g->directed);
         XBFS_CUDA(g, cudaGetLastError());
     }
     if (ds) {
@@ -170,6 +190,75 @@ xbfs_status pack_edges(xbfs_graph* g, const void* src, const void* dst, long lon
         cudaFree(ds);
         cudaFree(dd);
     }
+    return XBFS_OK;
+}
+
+// Directed graphs (f4): the in-arc CSR (in_row_ptr, in_col) of the out-arc CSR just
+// built, rows id-sorted; the bottom-up steps search it.
+xbfs_status build_transpose(xbfs_graph* g, int nb) {
+    const long long n = g->n, a = g->arcs;
+    XBFS_CUDA(g, cudaMalloc(&g->in_row_ptr, (n + 1) * sizeof(long long)));
+    XBFS_CUDA(g, cudaMalloc(&g->in_col, std::max<long long>(a, 1) * sizeof(int)));
+    if (a == 0) {
+        k_fill_rowptr<<<grid_for(n + 1), kB, 0, g->stream>>>(g->in_row_ptr, n, 0);
+        XBFS_CUDA(g, cudaGetLastError());
+        return XBFS_OK;
+    }
+    unsigned long long *k0 = nullptr, *k1 = nullptr;
+    XBFS_CUDA(g, cudaMalloc(&k0, a * sizeof(unsigned long long)));
+    XBFS_CUDA(g, cudaMalloc(&k1, a * sizeof(unsigned long long)));
+    k_transpose_keys<<<grid_for(a), kB, 0, g->stream>>>(g->row_ptr, g->col, n, a, nb, k0);
+    XBFS_CUDA(g, cudaGetLastError());
+    cub::DoubleBuffer<unsigned long long> db(k0, k1);
+    size_t tb = 0;
+    XBFS_CUDA(g, cub::DeviceRadixSort::SortKeys(nullptr, tb, db, a, 0, 2 * nb, g->stream));
+    void* tmp = nullptr;
+    XBFS_CUDA(g, cudaMalloc(&tmp, tb));
+    XBFS_CUDA(g, cub::DeviceRadixSort::SortKeys(tmp, tb, db, a, 0, 2 * nb, g->stream));
+    k_split_keys<<<grid_for(a), kB, 0, g->stream>>>(db.Current(), a, n, nb, g->in_col, g->in_row_ptr);
+    XBFS_CUDA(g, cudaGetLastError());
+    XBFS_CUDA(g, cudaStreamSynchronize(g->stream));
+    cudaFree(tmp);
+    cudaFree(k0);
+    cudaFree(k1);
+    return XBFS_OK;
+}
+
+// Re-arrange the rows of (rp, *colp) by mode (1: neighbour out-degree descending,
+// ties id ascending; 0: id order).  *colp may be replaced by the sort's buffer.
+xbfs_status reorder_rows(xbfs_graph* g, const long long* rp, int** colp, int mode) {
+    const long long a = g->arcs, n = g->n;
+    const int nb = std::max(1, bitlen((unsigned long long)(n - 1)));
+    const int db = std::max(1, bitlen((unsigned long long)g->max_deg));
+    const int low = mode == 1 ? db : nb;
+    const int shift = low;
+    const int total_bits = nb + low;
+    if (total_bits > 64) return set_error(XBFS_ERR_UNSUPPORTED, "reorder key does not fit in 64 bits");
+    unsigned long long *k0 = nullptr, *k1 = nullptr;
+    int* c1 = nullptr;
+    XBFS_CUDA(g, cudaMalloc(&k0, a * sizeof(unsigned long long)));
+    XBFS_CUDA(g, cudaMalloc(&k1, a * sizeof(unsigned long long)));
+    XBFS_CUDA(g, cudaMalloc(&c1, a * sizeof(int)));
+    k_reorder_keys<<<grid_for(a), kB, 0, g->stream>>>(rp, *colp, n, a, mode, shift,
+                                                      (unsigned long long)g->max_deg, k0, g->row_ptr);
+    XBFS_CUDA(g, cudaGetLastError());
+    cub::DoubleBuffer<unsigned long long> dk(k0, k1);
+    cub::DoubleBuffer<int> dv(*colp, c1);
+    size_t tb = 0;
+    XBFS_CUDA(g, cub::DeviceRadixSort::SortPairs(nullptr, tb, dk, dv, a, 0, total_bits, g->stream));
+    void* tmp = nullptr;
+    XBFS_CUDA(g, cudaMalloc(&tmp, tb));
+    XBFS_CUDA(g, cub::DeviceRadixSort::SortPairs(tmp, tb, dk, dv, a, 0, total_bits, g->stream));
+    XBFS_CUDA(g, cudaStreamSynchronize(g->stream));
+    cudaFree(tmp);
+    if (dv.Current() != *colp) {
+        cudaFree(*colp);
+        *colp = dv.Current();
+    } else {
+        cudaFree(c1);
+    }
+    cudaFree(k0);
+    cudaFree(k1);
     return XBFS_OK;
 }
 
@@ -202,6 +291,12 @@ xbfs_status alloc_work(xbfs_graph* g) {
 
 using namespace xbfs;
 
+#define XBFS_TRY_B(expr)                        \
+    do {                                        \
+        xbfs_status _s = (expr);                \
+        if (_s != XBFS_OK) return _s;           \
+    } while (0)
+
 extern "C" xbfs_status xbfs_build_csr(const void* src, const void* dst, int64_t m, int64_t n,
                                       const xbfs_build_opts* opts, xbfs_graph** out) {
     if (!out) return set_error(XBFS_ERR_INVALID_ARG, "xbfs_build_csr: out is NULL");
@@ -232,6 +327,7 @@ extern "C" xbfs_status xbfs_build_csr(const void* src, const void* dst, int64_t 
     XBFS_CUDA(g, cudaDeviceGetAttribute(&g->num_sms, cudaDevAttrMultiProcessorCount, g->device));
     g->n = n;
     g->m_input = m;
+    g->directed = o.directed ? 1 : 0;
     const int nb = std::max(1, bitlen((unsigned long long)(n - 1)));
     const long long nkeys = 2 * m;
 
@@ -314,24 +410,43 @@ extern "C" xbfs_status xbfs_build_csr(const void* src, const void* dst, int64_t 
         XBFS_CUDA(g, cudaGetLastError());
     }
     cudaFree(bad);
+    if (g->directed) {
+        xbfs_status st = build_transpose(g, nb);
+        if (st != XBFS_OK) return st;
+    }
 
     const long long words = (n + 31) / 32;
     XBFS_CUDA(g, cudaMalloc(&g->nonisolated, words * sizeof(unsigned int)));
     xbfs_status s = alloc_work(g);
     if (s != XBFS_OK) return s;
+    unsigned long long facts[2];
     XBFS_CUDA(g, cudaMemsetAsync(g->red_scratch, 0, 8 * sizeof(unsigned long long), g->stream));
     k_degree_facts<<<grid_for(words), kB, 0, g->stream>>>(g->row_ptr, n, words, g->nonisolated, g->red_scratch);
     XBFS_CUDA(g, cudaGetLastError());
-    unsigned long long facts[2];
     XBFS_CUDA(g, cudaMemcpyAsync(facts, g->red_scratch, sizeof(facts), cudaMemcpyDeviceToHost, g->stream));
     XBFS_CUDA(g, cudaStreamSynchronize(g->stream));
     g->nonisolated_count = (long long)facts[0];
-    g->max_deg = (int)facts[1];
+    g->max_deg = (int)facts[1];   // max (out-)degree: reorder key width, selector facts
+    if (g->directed) {
+        // BU candidates of a directed graph: vertices with an in-arc (reading R-9)
+        XBFS_CUDA(g, cudaMemsetAsync(g->red_scratch, 0, 8 * sizeof(unsigned long long), g->stream));
+        k_degree_facts<<<grid_for(words), kB, 0, g->stream>>>(g->in_row_ptr, n, words, g->nonisolated,
+                                                              g->red_scratch);
+        XBFS_CUDA(g, cudaGetLastError());
+        XBFS_CUDA(g, cudaMemcpyAsync(facts, g->red_scratch, sizeof(facts), cudaMemcpyDeviceToHost, g->stream));
+        XBFS_CUDA(g, cudaStreamSynchronize(g->stream));
+        g->nonisolated_count = (long long)facts[0];
+    }
     XBFS_CUDA(g, cudaMalloc(&g->head, n * sizeof(unsigned long long)));
     XBFS_CUDA(g, cudaMalloc(&g->head32, std::max<long long>(n, 1) * sizeof(unsigned)));
     g->idbits = std::max(1, bitlen((unsigned long long)(n - 1)));
     k_head<<<grid_for(n), kB, 0, g->stream>>>(g->row_ptr, g->col, n, g->head, g->head32, g->idbits);
     XBFS_CUDA(g, cudaGetLastError());
+    if (g->directed) {
+        XBFS_CUDA(g, cudaMalloc(&g->in_head32, std::max<long long>(n, 1) * sizeof(unsigned)));
+        k_head<<<grid_for(n), kB, 0, g->stream>>>(g->in_row_ptr, g->in_col, n, nullptr, g->in_head32, g->idbits);
+        XBFS_CUDA(g, cudaGetLastError());
+    }
     if ((unsigned long long)arcs >= (1ull << g->dbits))
         return set_error(XBFS_ERR_INVALID_ARG, "graph too large for the packed queue counter");
     guard.keep = true;
@@ -345,38 +460,13 @@ extern "C" xbfs_status xbfs_reorder(xbfs_graph* g, int32_t mode) {
     if (g->poisoned) return set_error(XBFS_ERR_STATE, "handle poisoned by an earlier failure");
     if (g->arcs == 0) { g->reorder_mode = mode; return XBFS_OK; }
     XBFS_CUDA(g, cudaSetDevice(g->device));
-    const long long a = g->arcs, n = g->n;
-    const int nb = std::max(1, bitlen((unsigned long long)(n - 1)));
-    const int db = std::max(1, bitlen((unsigned long long)g->max_deg));
-    const int low = mode == 1 ? db : nb;
-    const int shift = low;
-    const int total_bits = nb + low;
-    if (total_bits > 64) return set_error(XBFS_ERR_UNSUPPORTED, "reorder key does not fit in 64 bits");
-    unsigned long long *k0 = nullptr, *k1 = nullptr;
-    int* c1 = nullptr;
-    XBFS_CUDA(g, cudaMalloc(&k0, a * sizeof(unsigned long long)));
-    XBFS_CUDA(g, cudaMalloc(&k1, a * sizeof(unsigned long long)));
-    XBFS_CUDA(g, cudaMalloc(&c1, a * sizeof(int)));
-    k_reorder_keys<<<grid_for(a), kB, 0, g->stream>>>(g->row_ptr, g->col, n, a, mode, shift,
-                                                      (unsigned long long)g->max_deg, k0);
-    XBFS_CUDA(g, cudaGetLastError());
-    cub::DoubleBuffer<unsigned long long> dk(k0, k1);
-    cub::DoubleBuffer<int> dv(g->col, c1);
-    size_t tb = 0;
-    XBFS_CUDA(g, cub::DeviceRadixSort::SortPairs(nullptr, tb, dk, dv, a, 0, total_bits, g->stream));
-    void* tmp = nullptr;
-    XBFS_CUDA(g, cudaMalloc(&tmp, tb));
-    XBFS_CUDA(g, cub::DeviceRadixSort::SortPairs(tmp, tb, dk, dv, a, 0, total_bits, g->stream));
-    XBFS_CUDA(g, cudaStreamSynchronize(g->stream));
-    cudaFree(tmp);
-    if (dv.Current() != g->col) {
-        cudaFree(g->col);
-        g->col = dv.Current();
-    } else {
-        cudaFree(c1);
+    const long long n = g->n;
+    XBFS_TRY_B(reorder_rows(g, g->row_ptr, &g->col, mode));
+    if (g->directed) {
+        XBFS_TRY_B(reorder_rows(g, g->in_row_ptr, &g->in_col, mode));
+        k_head<<<grid_for(n), kB, 0, g->stream>>>(g->in_row_ptr, g->in_col, n, nullptr, g->in_head32, g->idbits);
+        XBFS_CUDA(g, cudaGetLastError());
     }
-    cudaFree(k0);
-    cudaFree(k1);
     k_head<<<grid_for(n), kB, 0, g->stream>>>(g->row_ptr, g->col, n, g->head, g->head32, g->idbits);
     XBFS_CUDA(g, cudaGetLastError());
     XBFS_CUDA(g, cudaStreamSynchronize(g->stream));

@@ -123,6 +123,12 @@ struct KArgs {
     long long arcs;         // A
     int dbits;              // low bits of qctr holding the degree sum
     int track_max;          // keep qmax (frontier max degree) for the small-mode gate
+    // the CSR bottom-up steps search: the same as row_ptr/col/head32 on a symmetric
+    // graph, the transposed (in-arc) CSR on a directed one (reading R-9)
+    const long long* bu_row_ptr;
+    const int* bu_col;
+    const unsigned* bu_head32;
+    int directed;
 };
 
 }  // namespace xbfs
@@ -139,7 +145,12 @@ struct xbfs_graph {
     long long* row_ptr = nullptr;
     int* col = nullptr;
     int* tcount = nullptr;
-    unsigned int* nonisolated = nullptr;
+    unsigned int* nonisolated = nullptr; // BU candidates: degree > 0 (in-degree > 0 when directed)
+    // directed graphs (f4): transposed CSR searched by bottom-up steps
+    int directed = 0;
+    long long* in_row_ptr = nullptr;
+    int* in_col = nullptr;
+    unsigned* in_head32 = nullptr;
     unsigned long long* head = nullptr;  // deg << 32 | col[row_ptr[v]] (rebuilt by every reorder)
     unsigned* head32 = nullptr;          // the same in 4 bytes (degree capped, see k_head)
     int idbits = 32;

@@ -642,6 +642,7 @@ xbfs_status xbfs_dist_build(const void* src, const void* dst, int64_t m, int64_t
     if (opts) o = *opts;
     if (o.id_bytes == 0) o.id_bytes = 4;
     if (o.id_bytes != 4 && o.id_bytes != 8) return set_error(XBFS_ERR_INVALID_ARG, "id_bytes must be 4 or 8");
+    if (o.directed) return set_error(XBFS_ERR_UNSUPPORTED, "directed graphs are single-GPU only (xbfs_build_csr)");
     xbfs_dist* d = new (std::nothrow) xbfs_dist();
     if (!d) return set_error(XBFS_ERR_OUT_OF_MEMORY, "host allocation failed");
     if (o.device >= 0) {

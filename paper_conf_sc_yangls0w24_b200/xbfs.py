@@ -35,7 +35,8 @@ class XbfsError(RuntimeError):
 
 class BuildOpts(ctypes.Structure):
     _fields_ = [("device", ctypes.c_int32), ("id_bytes", ctypes.c_int32), ("stream", ctypes.c_void_p),
-                ("edges_on_device", ctypes.c_int32), ("keep_duplicates", ctypes.c_int32)]
+                ("edges_on_device", ctypes.c_int32), ("keep_duplicates", ctypes.c_int32),
+                ("directed", ctypes.c_int32)]
 
 
 class RunOpts(ctypes.Structure):
@@ -257,7 +258,8 @@ class Graph:
     ``src``/``dst``: torch tensors (cuda or cpu) or numpy arrays of uint32/int32
     or int64 vertex ids."""
 
-    def __init__(self, src, dst, num_vertices: int, device: int | None = None, stream=None, reorder: bool = True):
+    def __init__(self, src, dst, num_vertices: int, device: int | None = None, stream=None, reorder: bool = True,
+                 directed: bool = False):
         import torch
         if isinstance(src, np.ndarray):
             id_bytes = src.dtype.itemsize
@@ -274,7 +276,9 @@ class Graph:
         if stream is None:
             stream = torch.cuda.current_stream(device).cuda_stream
         self.device = device
-        o = BuildOpts(device=device, id_bytes=id_bytes, stream=stream, edges_on_device=on_dev, keep_duplicates=0)
+        o = BuildOpts(device=device, id_bytes=id_bytes, stream=stream, edges_on_device=on_dev, keep_duplicates=0,
+                      directed=int(bool(directed)))
+        self.directed = bool(directed)
         m = int(src.shape[0])
         self._h = xbfs_build_csr(src, dst, m, num_vertices, o)
         self.n, self.arcs, self.m_input, self.max_degree = xbfs_graph_info(self._h)

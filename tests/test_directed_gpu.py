@@ -1,0 +1,154 @@
+"""GPU parity for directed graphs (reading R-9): the CUDA path
+through the C ABI against the oracle's out-arc CSR, textbook BFS and arc-wise
+Graph500 validation.  Levels must match BIT-EXACTLY; parents must validate;
+the per-level counters (|F_k|, edgesF_k over OUT-degrees), vertices reached,
+arcs traversed and Graph500 m must equal the oracle's.  Every strategy is
+forced on every level besides the adaptive selector, so the in-arc bottom-up
+search is checked on its own."""
+import numpy as np
+import pytest
+
+import oracle
+from paper_conf_sc_yangls0w24_b200 import synth
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+MODES = [dict(), dict(force_strategy=0), dict(force_strategy=1), dict(force_strategy=2),
+         dict(alpha=0.005), dict(alpha=0.3, grow=1.0, ratio_min=0.0), dict(bu_stay=0.0),
+         dict(driver=3, force_strategy=2)]
+
+
+@pytest.fixture(scope="module")
+def xb():
+    from paper_conf_sc_yangls0w24_b200 import xbfs
+    return xbfs
+
+
+def _dev(a):
+    return torch.from_numpy(np.ascontiguousarray(a).view(np.int32)).cuda()
+
+
+def _check(g, og, src, dst, root, **opts):
+    level, parent, st = g.run(int(root), stats=True, **opts)
+    lv, pa = level.cpu().numpy(), parent.cpu().numpy()
+    ref, _, nl = oracle.bfs(og, int(root))
+    assert np.array_equal(lv, ref), f"levels differ (root {root}, {opts})"
+    assert oracle.validate_directed(og, src, dst, int(root), lv, pa) == 0, f"validation (root {root}, {opts})"
+    fs, fe = oracle.level_stats(og, ref)
+    assert st.num_levels == nl
+    cap = len(st.frontier_vertices)
+    assert st.frontier_vertices == fs.tolist()[:cap]
+    assert st.frontier_edges == fe.tolist()[:cap]
+    assert st.vertices_reached == int((ref >= 0).sum())
+    assert st.arcs_traversed == int(fe.sum())
+    assert st.input_edges_traversed == oracle.input_edges(src, ref)
+    if "force_strategy" in opts and nl > 1:
+        assert set(st.strategy) == {opts["force_strategy"]}
+    return st
+
+
+def _one_way_grid(w, h):
+    """Arcs right and down only: from (r, c) the reachable set is the lower-right
+    quadrant at Manhattan distance."""
+    v = np.arange(w * h).reshape(h, w)
+    right = np.stack([v[:, :-1].ravel(), v[:, 1:].ravel()], 1)
+    down = np.stack([v[:-1, :].ravel(), v[1:, :].ravel()], 1)
+    e = np.concatenate([right, down]).astype(np.uint32)
+    return e[:, 0].copy(), e[:, 1].copy(), w * h
+
+
+@pytest.mark.parametrize("scale", [10, 14])
+def test_directed_csr_bit_exact(xb, scale):
+    src, dst, n = synth.kronecker(scale, seed=4)
+    og = oracle.build_csr_directed(n, src, dst)
+    g = xb.Graph(_dev(src), _dev(dst), n, reorder=False, directed=True)
+    rp, col = g.csr()
+    assert g.arcs == og.arcs
+    assert np.array_equal(rp, og.row_ptr) and np.array_equal(col[: og.arcs], og.col)
+    g.reorder(1)
+    r = oracle.reorder(og)
+    rp, col = g.csr()
+    assert np.array_equal(col[: og.arcs], r.col)
+    g.close()
+
+
+@pytest.mark.parametrize("scale", [12, 15])
+def test_directed_kronecker(xb, scale):
+    src, dst, n = synth.kronecker(scale, seed=5)
+    og = oracle.build_csr_directed(n, src, dst)
+    g = xb.Graph(_dev(src), _dev(dst), n, directed=True)
+    roots = synth.roots(n, src, dst, 3)
+    seen_bu = False
+    for root in roots:
+        for opts in MODES:
+            st = _check(g, og, src, dst, root, **opts)
+            seen_bu |= 2 in st.strategy
+    assert seen_bu
+    g.close()
+
+
+def test_directed_random_with_sources_and_sinks(xb):
+    """Sparse random arcs: many vertices have no in-arc (never BU candidates) or
+    no out-arc; roots include a pure source and a pure sink."""
+    rng = np.random.default_rng(9)
+    n = 20000
+    e = rng.integers(0, n, size=(3 * n, 2)).astype(np.uint32)
+    src, dst = e[:, 0].copy(), e[:, 1].copy()
+    og = oracle.build_csr_directed(n, src, dst)
+    indeg = np.bincount(dst[src != dst], minlength=n)
+    outdeg = og.degree()
+    pure_src = int(np.flatnonzero((indeg == 0) & (outdeg > 0))[0])
+    pure_sink = int(np.flatnonzero((indeg > 0) & (outdeg == 0))[0])
+    g = xb.Graph(src, dst, n, directed=True)
+    for root in (int(src[0]), pure_src, pure_sink):
+        for opts in MODES:
+            _check(g, og, src, dst, root, **opts)
+    g.close()
+
+
+def test_directed_one_way_grid_and_cycle(xb):
+    src, dst, n = _one_way_grid(96, 80)
+    og = oracle.build_csr_directed(n, src, dst)
+    g = xb.Graph(src, dst, n, directed=True)
+    for root in (0, 96 * 40 + 50):
+        for opts in MODES:
+            _check(g, og, src, dst, root, **opts)
+    lv, _, _ = g.run(0)
+    r, c = np.divmod(np.arange(n), 96)
+    assert np.array_equal(lv.cpu().numpy(), r + c)       # closed form from the corner
+    g.close()
+    # directed cycle: N levels, one vertex each (deep-path driver case)
+    n = 3000
+    src = np.arange(n, dtype=np.uint32)
+    dst = ((src + 1) % n).astype(np.uint32)
+    og = oracle.build_csr_directed(n, src, dst)
+    g = xb.Graph(src, dst, n, directed=True)
+    for opts in (dict(), dict(force_strategy=2)):
+        st = _check(g, og, src, dst, 17, **opts)
+        assert st.num_levels == n
+    g.close()
+
+
+def test_directed_unsupported_modes(xb):
+    src, dst, n = synth.kronecker(8, seed=1)
+    g = xb.Graph(src, dst, n, directed=True)
+    for opts in (dict(driver=1), dict(driver=2), dict(lookahead=1)):
+        with pytest.raises(xb.XbfsError) as ei:
+            g.run(int(src[0]), **opts)
+        assert ei.value.status == xb.XBFS_ERR_UNSUPPORTED
+    g.run(int(src[0]))                                     # the handle still works
+    g.close()
+
+
+def test_symmetric_input_directed_equals_undirected(xb):
+    """Both arcs of every tuple given as a directed graph = the undirected graph."""
+    src, dst, n = synth.kronecker(12, seed=6)
+    s2 = np.concatenate([src, dst]); d2 = np.concatenate([dst, src])
+    gd = xb.Graph(s2, d2, n, directed=True)
+    gu = xb.Graph(src, dst, n)
+    for root in synth.roots(n, src, dst, 3):
+        ld, _, _ = gd.run(int(root))
+        lu, _, _ = gu.run(int(root))
+        assert torch.equal(ld, lu)
+    gd.close(); gu.close()
