@@ -45,6 +45,8 @@ CONFIGS = {
     "s25": dict(kind="kron", scale=25, edgefactor=16),
     "s27": dict(kind="kron", scale=27, edgefactor=16),   # BASELINE config 4's graph (p = 1 point)
     "grid": dict(kind="grid", width=4096, height=4096),
+    # SURVEY f4 / reading R-9: the same Kronecker tuples taken as arcs i -> j (directed BFS)
+    "s24d": dict(kind="kron", scale=24, edgefactor=16, directed=True),
 }
 GRAPH_SEED, ROOT_SEED = 1, 2
 
@@ -52,7 +54,7 @@ GRAPH_SEED, ROOT_SEED = 1, 2
 def workload_name(cfg_name: str) -> str:
     c = CONFIGS[cfg_name]
     if c["kind"] == "kron":
-        return f"graph500-kronecker-s{c['scale']}-ef{c['edgefactor']}"
+        return f"graph500-kronecker-s{c['scale']}-ef{c['edgefactor']}" + ("-directed" if c.get("directed") else "")
     return f"grid-{c['width']}x{c['height']}"
 
 
@@ -219,14 +221,27 @@ def run_ours(args):
 
     stream = torch.cuda.current_stream(dev)
     t0 = time.time()
+    directed = bool(CONFIGS[args.config].get("directed"))
     g = Graph(torch.from_numpy(src.view(np.int32)), torch.from_numpy(dst.view(np.int32)), n, device=local,
-              stream=stream.cuda_stream, reorder=False)
+              stream=stream.cuda_stream, reorder=False, directed=directed)
     torch.cuda.synchronize()
     t_build = time.time() - t0
     t0 = time.time()
     g.reorder(1)
     torch.cuda.synchronize()
     t_reorder = time.time() - t0
+    root_rule = "Graph500 (seeded, touching a non-self-loop tuple)"
+    if directed:
+        # R-9 root recipe: seeded candidates whose forward reach is >= 1 % of N (the giant
+        # out-component; a root whose out-arcs lead to a sink reaches a handful of vertices),
+        # screened with untimed runs of this library
+        cand = pick_roots(args.config, n, src, dst, 4 * total_roots)
+        keep = [int(r) for r in cand if g.run(int(r), stats=True)[2].vertices_reached >= n // 100]
+        roots = np.resize(np.asarray(keep, dtype=np.int64), total_roots)
+        warm = roots[: args.warmup]
+        mine = roots[args.warmup + rank * args.steps: args.warmup + (rank + 1) * args.steps]
+        root_rule = f"directed: seeded candidates with forward reach >= N/100 ({len(keep)} of {len(cand)} kept)"
+        args.profile_roots = 0       # per-launch profiling runs the host-loop driver (undirected only)
     level = torch.empty(n, dtype=torch.int32, device=dev)
     parent = torch.empty(n, dtype=torch.int32, device=dev)
     flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
@@ -258,7 +273,7 @@ def run_ours(args):
                          "".join("FSB"[s] for s in st.strategy)))
         launches += st.kernel_launches
         lb = metrics.bfs_level_bytes(n, st.strategy, st.frontier_vertices, st.frontier_edges, st.unvisited,
-                                     st.bu_probes)
+                                     st.bu_probes, directed=directed)
         alg_bytes += metrics.bytes_init(n) + sum(lb)
         for s_, ms_, b_ in zip(st.strategy, st.level_ms, lb):
             ph = phase.setdefault("FSB"[s_], [0, 0.0, 0])
@@ -400,6 +415,7 @@ def run_ours(args):
         "config": {"workload": workload_name(args.config), "n_vertices": n, "input_edges": int(src.shape[0]),
                    "arcs": g.arcs, "roots_per_gpu": args.steps, "l2_flush": "512 MiB write before every timed BFS",
                    "reorder": "degree-desc (P:L153)", "alpha": opts.get("alpha", default_alpha()),
+                   "roots": root_rule,
                    "bu_stay": opts.get("bu_stay", 1.0),
                    "driver": {0: "persistent (auto)", 1: "host loop", 2: "CUDA-graph loop",
                               3: "persistent"}[args.driver],
@@ -440,7 +456,7 @@ def cpu_baseline(args, src, dst, n, roots, m_of=None, budget_s=None):
     import oracle
     budget_s = args.cpu_budget if budget_s is None else budget_s
     t0 = time.time()
-    og = oracle.build_csr(n, src, dst)
+    og = (oracle.build_csr_directed if CONFIGS[args.config].get("directed") else oracle.build_csr)(n, src, dst)
     t_csr = time.time() - t0
     teps, used, spent = [], [], 0.0
     for r in roots:
@@ -469,15 +485,21 @@ def run_reference(args):
     import oracle
     from paper_conf_sc_yangls0w24_b200 import metrics
     src, dst, n = make_graph(args.config, pinned=False)
-    roots = pick_roots(args.config, n, src, dst, args.warmup + args.steps * world)
-    og = oracle.build_csr(n, src, dst)
+    directed = bool(CONFIGS[args.config].get("directed"))
+    roots = pick_roots(args.config, n, src, dst, 4 * (args.warmup + args.steps * world) if directed
+                       else args.warmup + args.steps * world)
+    og = (oracle.build_csr_directed if directed else oracle.build_csr)(n, src, dst)
     for r in roots[: args.warmup]:
         oracle.bfs(og, int(r))
     teps, times = [], []
-    for r in roots[args.warmup: args.warmup + args.steps]:
+    for r in roots[args.warmup:]:
+        if len(teps) == args.steps:
+            break
         t1 = time.perf_counter()
         lv, _, _ = oracle.bfs(og, int(r))
         dt = time.perf_counter() - t1
+        if directed and int((lv >= 0).sum()) < n // 100:
+            continue                 # the R-9 root rule (forward reach >= N/100), as in our arm
         teps.append(oracle.input_edges(src, lv) / dt)
         times.append(dt)
     value = metrics.harmonic_mean(teps) / 1e9

@@ -266,7 +266,7 @@ __device__ __forceinline__ void seed_body(const KArgs& a, int* level, int* paren
     st->fprev = 0;
     st->unvisited = nonisolated_count - (s_cand ? 1 : 0);
     for (int i = 0; i < 3; ++i) {
-        st->acc_found[i] = st->acc_edges[i] = st->acc_probes[i] = 0;
+        st->acc_found[i] = st->acc_edges[i] = st->acc_probes[i] = st->acc_zero[i] = 0;
         st->acc_la_found[i] = st->acc_la_edges[i] = 0;
     }
     st->reached = 0;
@@ -310,6 +310,7 @@ __device__ __forceinline__ void select_step(const KArgs& a, SelState& s, bool lo
         const unsigned long long q = __ldcg(&st->qctr[(k + 1) % 3]);
         nf = (long long)(q >> a.dbits);
         ne = (long long)(q & ((1ull << a.dbits) - 1ull));
+        if (a.directed) nf += (long long)__ldcg(&st->acc_zero[k % 3]);   // unqueued sinks
         s.queue_valid = 1;
     }
     // look-ahead (persistent driver): vertices of F_{k+1} that BU step k-1 already
@@ -415,6 +416,7 @@ __device__ void select_body(const KArgs& a) {
     st->qctr[(k + 2) % 3] = 0;   // counter of the queue built during level k+1
     st->qmax[(k + 2) % 3] = 0;
     st->acc_found[(k + 1) % 3] = st->acc_edges[(k + 1) % 3] = st->acc_probes[(k + 1) % 3] = 0;
+    st->acc_zero[(k + 1) % 3] = 0;
     st->acc_la_found[(k + 1) % 3] = st->acc_la_edges[(k + 1) % 3] = 0;
     sel_store(st, s);
     mirror_host(a, st);
@@ -449,7 +451,8 @@ using TdSmem = TdSmemT<1>;
 #endif
 constexpr long long kSfPrecheckMin = XBFS_SF_PRECHECK_MIN;   // edgesF_k above which SF probes before claiming
 
-template <int MODE, int THREADS, int TPT = 1>
+// DIR: directed graph (f4, R-9): out-degree-0 winners are counted, not queued.
+template <int MODE, int THREADS, int TPT = 1, bool DIR = false>
 __device__ __forceinline__ void td_expand_body(const KArgs& a, int k, int* __restrict__ level,
                                                int* __restrict__ parent, TdSmemT<TPT>& sm, long long Fs = -1,
                                                long long Ts = -1) {
@@ -542,6 +545,16 @@ __device__ __forceinline__ void td_expand_body(const KArgs& a, int k, int* __res
             }
 #pragma unroll
             for (int i = 0; i < R; ++i) deg[i] -= rs[i];
+            if constexpr (DIR) {
+                int zc = 0;     // winners without out-arcs (directed sinks) are counted, not queued
+#pragma unroll
+                for (int i = 0; i < R; ++i)
+                    if (win[i] && deg[i] == 0) { ++zc; win[i] = false; }
+                if (__any_sync(FULL, zc)) {
+                    zc = __reduce_add_sync(FULL, (unsigned)zc);
+                    if ((threadIdx.x & 31) == 0) atomicAdd(&a.st->acc_zero[k % 3], (unsigned long long)zc);
+                }
+            }
             enqueue_warp_multi<R>(win, v, rs, deg, &a.st->qctr[(k + 1) % 3], lmax, a.dbits, a.qv[ob],
                                   a.qoff[ob], a.qdelta[ob], a.tile_first[ob]);
         } else {
@@ -640,13 +653,16 @@ __device__ __forceinline__ void generate_body(const KArgs& a, int k, int role) {
         const long long w = w0 + lane;
         unsigned word = w < a.words ? __ldcg(bm + w) : 0u;
         if (role == 1 && word) a.visited[w] = __ldcg(a.visited + w) | word;
-        // pass 1: count and degree sum of this lane's vertices
-        const int cnt = __popc(word);
+        // pass 1: count and degree sum of this lane's vertices; vertices without
+        // (out-)arcs are not queued (directed sinks: nothing to expand, and a tile's
+        // queue range must stay within its arcs)
+        int cnt = 0;
         long long dsum = 0;
         for (unsigned b = word; b; b &= b - 1) {
             const long long v = w * 32 + __ffs(b) - 1;
             const long long d = a.row_ptr[v + 1] - a.row_ptr[v];
             dsum += d;
+            cnt += d > 0;
             gmax = max(gmax, (unsigned)d);
         }
         int ic = cnt;
@@ -672,6 +688,7 @@ __device__ __forceinline__ void generate_body(const KArgs& a, int k, int role) {
         for (unsigned b = word; b; b &= b - 1) {
             const long long v = w * 32 + __ffs(b) - 1;
             const long long rs = a.row_ptr[v], deg = a.row_ptr[v + 1] - rs;
+            if (deg == 0) continue;
             qv[slot] = (int)v;
             qoff[slot] = off;
             qdelta[slot] = rs - off;
@@ -698,7 +715,7 @@ __global__ __launch_bounds__(kGenThreads) void k_generate(KArgs a, int role) {
 // kp: where k lives (DevState or the persistent CTA's selector copy); it is
 // re-read for the epilogue instead of keeping k live across the traversal
 // (one register less: the per-level kernel runs at 48 without spills).
-template <int WARPS, bool LA, class Smem>
+template <int WARPS, bool LA, class Smem, bool DIR = false>
 __device__ __forceinline__ void bu_body(const KArgs& a, const int* kp, int* __restrict__ level,
                                         int* __restrict__ parent, Smem& sm, bool prefill) {
     int k = *(const volatile int*)kp;
@@ -715,10 +732,10 @@ __device__ __forceinline__ void bu_body(const KArgs& a, const int* kp, int* __re
     b.visited = a.visited;
     b.words = a.words;
     b.head = a.head;
-    b.head32 = a.bu_head32;          // in-arc CSR on a directed graph (f4, R-9)
+    b.head32 = DIR ? a.bu_head32 : a.head32;   // in-arc CSR on a directed graph (f4, R-9)
     b.idbits = a.idbits;
-    b.row_ptr = a.bu_row_ptr;
-    b.col = a.bu_col;
+    b.row_ptr = DIR ? a.bu_row_ptr : a.row_ptr;
+    b.col = DIR ? a.bu_col : a.col;
     b.level = level;
     b.parent = parent;
     b.lvl = lvl;
@@ -745,7 +762,7 @@ __device__ __forceinline__ void bu_body(const KArgs& a, const int* kp, int* __re
     // directed graph: the BU rows are in-arc rows, whose lengths are not the out-degrees
     // edgesF_{k+1} needs; the count pass (ss_count_body) that follows supplies |F_{k+1}|
     // and edgesF_{k+1} from the out-arc head[] instead
-    if (a.directed) found = edges = 0;
+    if (DIR) found = edges = 0;
     if (lane == 0 && (found | edges | probes)) {
         atomicAdd(&a.st->acc_found[k % 3], found);
         atomicAdd(&a.st->acc_edges[k % 3], edges);
@@ -981,7 +998,7 @@ __global__ void __cluster_dims__(kSmallCluster, 1, 1) __launch_bounds__(kSmallTh
         st->reached = reached;
         st->arcs_traversed = arcs_tr;
         st->prev_strategy = XBFS_SF;
-        for (int i = 0; i < 3; ++i) st->acc_found[i] = st->acc_edges[i] = st->acc_probes[i] = 0;
+        for (int i = 0; i < 3; ++i) st->acc_found[i] = st->acc_edges[i] = st->acc_probes[i] = st->acc_zero[i] = 0;
         st->fmaxdeg = fmaxdeg;
         st->advanced = st->mirror_host ? 0 : 1;   // graph driver: its k_select node only mirrors
         st->prev_small = 1;
@@ -1076,7 +1093,8 @@ union PersistSmem {
 
 // LA: the BU look-ahead variant (a separate instantiation, so the default kernel
 // carries none of its registers).
-template <bool LA>
+// DIR: directed graph (f4, reading R-9; also a separate instantiation).
+template <bool LA, bool DIR>
 __global__ __launch_bounds__(kPersistThreads, kPersistBlocks) void k_persist(
     KArgs a, int* __restrict__ level, int* __restrict__ parent, const unsigned int* __restrict__ nonisolated,
     long long nonisolated_count) {
@@ -1103,6 +1121,7 @@ __global__ __launch_bounds__(kPersistThreads, kPersistBlocks) void k_persist(
             a.st->qctr[(k + 2) % 3] = 0;
             a.st->qmax[(k + 2) % 3] = 0;
             a.st->acc_found[(k + 1) % 3] = a.st->acc_edges[(k + 1) % 3] = a.st->acc_probes[(k + 1) % 3] = 0;
+            a.st->acc_zero[(k + 1) % 3] = 0;
             a.st->acc_la_found[(k + 1) % 3] = a.st->acc_la_edges[(k + 1) % 3] = 0;
         }
         if (strat != XBFS_BU && !qvalid) {
@@ -1110,16 +1129,19 @@ __global__ __launch_bounds__(kPersistThreads, kPersistBlocks) void k_persist(
             grid_sync(bar, epoch);
         }
         if (strat == XBFS_SF) {
-            td_expand_body<XBFS_SF, kPersistThreads, XBFS_SF_TPT>(
-                a, k, level, parent, *reinterpret_cast<TdSmemT<XBFS_SF_TPT>*>(&sm.td), s.fsize, s.fedges);
+            // (directed: the queue holds |F_k| minus the sinks; read its own count)
+            td_expand_body<XBFS_SF, kPersistThreads, XBFS_SF_TPT, DIR>(
+                a, k, level, parent, *reinterpret_cast<TdSmemT<XBFS_SF_TPT>*>(&sm.td), DIR ? -1 : s.fsize,
+                s.fedges);
         } else if (strat == XBFS_SS) {
-            td_expand_body<XBFS_SS, kPersistThreads, XBFS_SS_TPT>(
-                a, k, level, parent, *reinterpret_cast<TdSmemT<XBFS_SS_TPT>*>(&sm.td), s.fsize, s.fedges);
+            td_expand_body<XBFS_SS, kPersistThreads, XBFS_SS_TPT, DIR>(
+                a, k, level, parent, *reinterpret_cast<TdSmemT<XBFS_SS_TPT>*>(&sm.td), DIR ? -1 : s.fsize,
+                s.fedges);
             grid_sync(bar, epoch);
             ss_count_body(a, k);
         } else {
-            bu_body<kPersistThreads / 32, LA>(a, &s.k, level, parent, sm.bu, s.prefill);
-            if (a.directed) {       // |F_{k+1}|, edgesF_{k+1} over out-arcs (see bu_body)
+            bu_body<kPersistThreads / 32, LA, decltype(sm.bu), DIR>(a, &s.k, level, parent, sm.bu, s.prefill);
+            if constexpr (DIR) {    // |F_{k+1}|, edgesF_{k+1} over out-arcs (see bu_body)
                 grid_sync(bar, epoch);
                 ss_count_body(a, k);
             }
@@ -1385,10 +1407,11 @@ xbfs_status build_loop_graph(xbfs_graph* g, int* level, int* parent) {
 }
 
 xbfs_status launch_persist(xbfs_graph* g, const KArgs& a, int* level, int* parent, bool lookahead) {
-    static int occ[2][64];
-    static bool init[2][64] = {{false}};
-    const int dev = g->device & 63, v = lookahead ? 1 : 0;
-    void* fn = lookahead ? (void*)k_persist<true> : (void*)k_persist<false>;
+    static int occ[3][64];
+    static bool init[3][64] = {{false}};
+    const int dev = g->device & 63, v = lookahead ? 1 : (g->directed ? 2 : 0);
+    void* fn = lookahead ? (void*)k_persist<true, false>
+                         : (g->directed ? (void*)k_persist<false, true> : (void*)k_persist<false, false>);
     const size_t smem = lookahead ? sizeof(PersistSmem<true>) : sizeof(PersistSmem<false>);
     if (!init[v][dev]) {
         XBFS_CUDA(g, cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));

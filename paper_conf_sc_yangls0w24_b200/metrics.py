@@ -91,7 +91,7 @@ def bytes_ss_count(n: int, found: int) -> int:
     return bitmap_bytes(n) + 8 * found
 
 
-def bfs_level_bytes(n: int, strategy, fv, fe, unvisited, probes):
+def bfs_level_bytes(n: int, strategy, fv, fe, unvisited, probes, directed: bool = False):
     """Algorithmic bytes of every level of one BFS given the strategies the
     selector took (the phases of the persistent kernel): SF and SS
     read a queue that exists after an SF level (No-Frontier-Generation) and is
@@ -111,10 +111,12 @@ def bfs_level_bytes(n: int, strategy, fv, fe, unvisited, probes):
             b += bytes_td_ss(n, fv[k], fe[k], found) + bytes_ss_count(n, found)
         else:
             b += bytes_bu(n, unvisited[k], probes[k], found)
+            if directed:     # in-arc rows do not give out-degrees: the count pass follows (R-9)
+                b += bytes_ss_count(n, found)
         out.append(b)
     return out
 
 
-def bfs_alg_bytes(n: int, strategy, fv, fe, unvisited, probes) -> int:
+def bfs_alg_bytes(n: int, strategy, fv, fe, unvisited, probes, directed: bool = False) -> int:
     """Init + every level: the algorithmic bytes of one persistent-kernel launch."""
-    return bytes_init(n) + sum(bfs_level_bytes(n, strategy, fv, fe, unvisited, probes))
+    return bytes_init(n) + sum(bfs_level_bytes(n, strategy, fv, fe, unvisited, probes, directed))

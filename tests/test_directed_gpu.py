@@ -152,3 +152,34 @@ def test_symmetric_input_directed_equals_undirected(xb):
         lu, _, _ = gu.run(int(root))
         assert torch.equal(ld, lu)
     gd.close(); gu.close()
+
+
+def test_directed_kronecker_s20_saturated_head(xb):
+    """Scale 20: head32 holds 20-bit ids, so in-degrees >= 4095 saturate and the
+    bottom-up resolves them from in_row_ptr (the s24 bench case has dmax = 255)."""
+    src, dst, n = synth.kronecker(20, seed=1)
+    og = oracle.build_csr_directed(n, src, dst)
+    g = xb.Graph(src, dst, n, directed=True)
+    for root in synth.roots(n, src, dst, 2):
+        for opts in (dict(), dict(force_strategy=2)):
+            _check(g, og, src, dst, root, **opts)
+    g.close()
+
+
+def test_directed_sinks_fill_a_tile(xb):
+    """Many out-degree-0 vertices discovered in one top-down level (a hub with
+    20000 arcs into sinks plus a few real rows): the queue holds only vertices
+    with arcs, so a 2048-arc tile never spans more entries than it has arcs."""
+    hub, nsink = 0, 20000
+    sinks = np.arange(1, nsink + 1)
+    chain = np.arange(nsink + 1, nsink + 50)
+    extra = sinks[::97]                       # a few of them do have out-arcs (into the chain)
+    src = np.concatenate([np.full(nsink, hub), np.full(chain.size, hub), chain[:-1], extra])
+    dst = np.concatenate([sinks, chain, chain[1:], nsink + 1 + np.arange(extra.size) % chain.size])
+    n = nsink + 50
+    src, dst = src.astype(np.uint32), dst.astype(np.uint32)
+    og = oracle.build_csr_directed(n, src, dst)
+    g = xb.Graph(src, dst, n, directed=True)
+    for opts in MODES:
+        _check(g, og, src, dst, hub, **opts)
+    g.close()
