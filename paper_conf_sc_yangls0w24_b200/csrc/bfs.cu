@@ -971,6 +971,7 @@ __global__ void __cluster_dims__(kSmallCluster, 1, 1) __launch_bounds__(kSmallTh
             rec.la_found = 0;
             rec.strategy = XBFS_SF;
             rec.pad = 0;
+            rec.t_ns = 0;            // (no %globaltimer stamps outside the persistent driver)
             a.log[k] = rec;
         }
         reached += fsize;

@@ -24,5 +24,21 @@ for name, (src, dst, n) in {"kron11": synth.kronecker(11, seed=3), "grid": synth
                     continue
                 lv, pa, st = g.run(int(root), stats=True, driver=drv, **opts)
     g.close()
+# SANITIZE_PERSIST=1: the persistent driver (3), undirected and directed (f4) graphs,
+# including a sink-heavy top-down level
+if os.environ.get("SANITIZE_PERSIST") == "1":
+    hub, ns = 0, 5000
+    sk = np.arange(1, ns + 1)
+    ch = np.arange(ns + 1, ns + 40)
+    s_src = np.concatenate([np.zeros(ns + ch.size, np.int64), ch[:-1]]).astype(np.uint32)
+    s_dst = np.concatenate([sk, ch, ch[1:]]).astype(np.uint32)
+    cases = [("kron11", synth.kronecker(11, seed=3), False), ("grid", synth.grid(33, 17, seed=1), False),
+             ("kron11d", synth.kronecker(11, seed=3), True), ("sinks", (s_src, s_dst, ns + 40), True)]
+    for name, (src, dst, n), directed in cases:
+        g = Graph(src, dst, n, directed=directed)
+        for root in list(synth.roots(n, src, dst, 2, root_seed=4)) + [0]:
+            for opts in (dict(), dict(force_strategy=0), dict(force_strategy=1), dict(force_strategy=2)):
+                g.run(int(root), stats=True, driver=3, **opts)
+        g.close()
 torch.cuda.synchronize()
 print("sanitize workload done")
