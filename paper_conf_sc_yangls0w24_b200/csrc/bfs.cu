@@ -178,8 +178,11 @@ __device__ __forceinline__ void mirror_host(const KArgs& a, const DevState* st) 
 }
 
 // ---------------------------------------------------------------- init
+// src >= 0 (persistent driver): the thread that fills the source's element writes
+// its seed values instead (level 0, parent = itself, visited and F_0 bits), so the
+// seed needs no barrier of its own after the fill.
 __device__ __forceinline__ void init_body(const KArgs& a, int* __restrict__ level, int* __restrict__ parent,
-                                          const unsigned int* __restrict__ nonisolated) {
+                                          const unsigned int* __restrict__ nonisolated, long long src = -1) {
     const long long tid = blockIdx.x * (long long)blockDim.x + threadIdx.x;
     const long long nth = (long long)gridDim.x * blockDim.x;
     const long long n4 = a.n / 4;
@@ -190,23 +193,41 @@ __device__ __forceinline__ void init_body(const KArgs& a, int* __restrict__ leve
     if ((((uintptr_t)level | (uintptr_t)parent) & 31) == 0) {
         // one 32-byte store per sector (STG.256)
         const long long n8 = a.n / 8;
+        const long long sc = src >= 0 ? src / 8 : -1;
         for (long long i = tid; i < n8; i += nth) {
             asm volatile("st.global.v8.b32 [%0], {%1,%1,%1,%1,%1,%1,%1,%1};" ::"l"(level + 8 * i), "r"(-1) : "memory");
             asm volatile("st.global.v8.b32 [%0], {%1,%1,%1,%1,%1,%1,%1,%1};" ::"l"(parent + 8 * i), "r"(-1) : "memory");
+            if (i == sc) { level[src] = 0; parent[src] = (int)src; }
         }
-        for (long long i = n8 * 8 + tid; i < a.n; i += nth) { level[i] = -1; parent[i] = -1; }
+        for (long long i = n8 * 8 + tid; i < a.n; i += nth) {
+            level[i] = i == src ? 0 : -1;
+            parent[i] = i == src ? (int)src : -1;
+        }
     } else
 #endif
     if ((((uintptr_t)level | (uintptr_t)parent) & 15) == 0) {
-        for (long long i = tid; i < n4; i += nth) { l4[i] = m1; p4[i] = m1; }
-        for (long long i = n4 * 4 + tid; i < a.n; i += nth) { level[i] = -1; parent[i] = -1; }
+        const long long sc = src >= 0 ? src / 4 : -1;
+        for (long long i = tid; i < n4; i += nth) {
+            l4[i] = m1;
+            p4[i] = m1;
+            if (i == sc) { level[src] = 0; parent[src] = (int)src; }
+        }
+        for (long long i = n4 * 4 + tid; i < a.n; i += nth) {
+            level[i] = i == src ? 0 : -1;
+            parent[i] = i == src ? (int)src : -1;
+        }
     } else {
-        for (long long i = tid; i < a.n; i += nth) { level[i] = -1; parent[i] = -1; }
+        for (long long i = tid; i < a.n; i += nth) {
+            level[i] = i == src ? 0 : -1;
+            parent[i] = i == src ? (int)src : -1;
+        }
     }
     // isolated vertices are pre-marked visited: never BU candidates (reading C-27)
+    const long long sw = src >= 0 ? src >> 5 : -1;
+    const unsigned sbit = src >= 0 ? 1u << (src & 31) : 0u;
     for (long long w = tid; w < a.words; w += nth) {
-        a.visited[w] = ~nonisolated[w];
-        a.fb[0][w] = 0;
+        a.visited[w] = ~nonisolated[w] | (w == sw ? sbit : 0u);
+        a.fb[0][w] = w == sw ? sbit : 0u;
         a.fb[1][w] = 0;
         a.fb[2][w] = 0;
         a.la[w] = 0;
@@ -233,16 +254,21 @@ __device__ int choose_strategy(const DevState* st, long long arcs, long long fsi
 
 // Seed the source (the source holds level 0) and reset the level state.
 // One thread.
-__device__ __forceinline__ void seed_body(const KArgs& a, int* level, int* parent, long long nonisolated_count) {
+// bits_done: init_body(src) already wrote the source's level/parent and bits.
+__device__ __forceinline__ void seed_body(const KArgs& a, int* level, int* parent, long long nonisolated_count,
+                                          const unsigned int* __restrict__ nonisolated, bool bits_done) {
     DevState* st = a.st;
     const long long s = st->source;   // per-run parameter copied in before init
     const long long rs = a.row_ptr[s], deg = a.row_ptr[s + 1] - rs;
-    level[s] = 0;
-    parent[s] = (int)s;
-    // the source was a BU candidate (counted in U_0) iff init left its visited bit clear
     const unsigned sbit = 1u << (s & 31);
-    const bool s_cand = !(atomicOr(a.visited + (s >> 5), sbit) & sbit);
-    atomicOr(a.fb[0] + (s >> 5), 1u << (s & 31));
+    // the source is a BU candidate (counted in U_0) iff it is not pre-set visited
+    const bool s_cand = (nonisolated[s >> 5] & sbit) != 0;
+    if (!bits_done) {
+        level[s] = 0;
+        parent[s] = (int)s;
+        atomicOr(a.visited + (s >> 5), sbit);
+        atomicOr(a.fb[0] + (s >> 5), sbit);
+    }
     a.qv[0][0] = (int)s;
     a.qoff[0][0] = 0;
     a.qdelta[0][0] = rs;
@@ -277,9 +303,10 @@ __device__ __forceinline__ void seed_body(const KArgs& a, int* level, int* paren
     st->strategy = choose_strategy(st, a.arcs, 1, 0, deg, st->unvisited, -1);
 }
 
-__global__ void k_seed(KArgs a, int* level, int* parent, long long nonisolated_count) {
+__global__ void k_seed(KArgs a, int* level, int* parent, long long nonisolated_count,
+                       const unsigned int* __restrict__ nonisolated) {
     count_launch(a.st);
-    seed_body(a, level, parent, nonisolated_count);
+    seed_body(a, level, parent, nonisolated_count, nonisolated, false);
     mirror_host(a, a.st);
 }
 
@@ -1105,13 +1132,12 @@ __global__ __launch_bounds__(kPersistThreads, kPersistBlocks) void k_persist(
     unsigned epoch = 0;
     unsigned* bar = &a.st->bar_count;
     count_launch(a.st);
-    init_body(a, level, parent, nonisolated);
+    // the source's entries are written by the fill itself and the seed state by one
+    // thread alongside it: one barrier for both
+    init_body(a, level, parent, nonisolated, *(const volatile long long*)&a.st->source);
+    if (blockIdx.x == 0 && threadIdx.x == 0) seed_body(a, level, parent, nonisolated_count, nonisolated, true);
     grid_sync(bar, epoch);
-    if (blockIdx.x == 0 && threadIdx.x == 0) {
-        seed_body(a, level, parent, nonisolated_count);
-        a.st->t_start = globaltimer();
-    }
-    grid_sync(bar, epoch);
+    if (blockIdx.x == 0 && threadIdx.x == 0) a.st->t_start = globaltimer();
     if (threadIdx.x == 0) sel_load(a.st, s);
     __syncthreads();
     for (;;) {
@@ -1346,7 +1372,7 @@ xbfs_status build_loop_graph(xbfs_graph* g, int* level, int* parent) {
         XBFS_TRY(add_kernel(g, top, &n_init, nullptr, (void*)k_init_fill, G.init, 256, args));
     }
     {
-        void* args[] = {&a, &level, &parent, &nic};
+        void* args[] = {&a, &level, &parent, &nic, &noniso};
         XBFS_TRY(add_kernel(g, top, &n_seed, &n_init, (void*)k_seed, 1, 1, args));
     }
     cudaGraphConditionalHandle h_while, h_switch;
@@ -1496,7 +1522,7 @@ static xbfs_status run_impl(xbfs_graph* g, int64_t source, int32_t* level, int32
     XBFS_LAUNCH(P, XBFS_K_INIT, -1,
                 (k_init_fill<<<G.init, 256, 0, g->stream>>>(a, level, parent, g->nonisolated)));
     XBFS_LAUNCH(P, XBFS_K_SEED, -1,
-                (k_seed<<<1, 1, 0, g->stream>>>(a, level, parent, g->nonisolated_count)));
+                (k_seed<<<1, 1, 0, g->stream>>>(a, level, parent, g->nonisolated_count, g->nonisolated)));
     XBFS_TRY(run_host_loop(g, a, level, parent, std::min<long long>(std::max(o.small_edges, 0), kSmallEdgesMax),
                            o.plan, o.plan ? std::max(o.plan_len, 0) : 0, P));
     XBFS_CUDA(g, cudaEventRecord(g->ev1, g->stream));
