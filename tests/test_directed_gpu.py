@@ -183,3 +183,19 @@ def test_directed_sinks_fill_a_tile(xb):
     for opts in MODES:
         _check(g, og, src, dst, hub, **opts)
     g.close()
+
+
+def test_bench_workload_s24d_full_size(xb):
+    """The directed bench workload at full size (bench.py --config s24d: the s24 Kronecker
+    tuples as arcs, 16.8 M vertices / 263 M arcs), persistent driver, default options:
+    levels bit-exact against the oracle's serial BFS, parents arc-validated, per-level
+    counters exact, one launch per BFS; roots are bench's candidates, including ones
+    whose forward reach is tiny (the bench screens those out; parity must hold anyway)."""
+    import bench
+    src, dst, n = bench.make_graph("s24d", pinned=False)
+    og = oracle.build_csr_directed(n, src, dst)
+    g = xb.Graph(_dev(src), _dev(dst), n, directed=True)
+    for root in bench.pick_roots("s24d", n, src, dst, 3):
+        st = _check(g, og, src, dst, root)
+        assert st.kernel_launches == 1
+    g.close()
