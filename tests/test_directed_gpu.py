@@ -199,3 +199,26 @@ def test_bench_workload_s24d_full_size(xb):
         st = _check(g, og, src, dst, root)
         assert st.kernel_launches == 1
     g.close()
+
+
+def test_directed_int64_device_edges_and_host_batch(xb):
+    """Directed build from int64 ids resident on the device (id_bytes 8,
+    edges_on_device 1) equals the oracle; the pipelined host-output batch call
+    returns every root's exact levels on it."""
+    src, dst, n = synth.kronecker(13, seed=8)
+    og = oracle.build_csr_directed(n, src, dst)
+    s64 = torch.from_numpy(src.astype(np.int64)).cuda()
+    d64 = torch.from_numpy(dst.astype(np.int64)).cuda()
+    g = xb.Graph(s64, d64, n, reorder=False, directed=True)
+    rp, col = g.csr()
+    assert np.array_equal(rp, og.row_ptr) and np.array_equal(col[: og.arcs], og.col)
+    g.reorder(1)
+    roots = [int(r) for r in synth.roots(n, src, dst, 4, root_seed=5)]
+    lh = np.empty(4 * n, np.int32)
+    ph = np.empty(4 * n, np.int32)
+    g.run_host_batch(roots, lh, ph)
+    for i, r in enumerate(roots):
+        ref, _, _ = oracle.bfs(og, r)
+        assert np.array_equal(lh[i * n:(i + 1) * n], ref)
+        assert oracle.validate_directed(og, src, dst, r, lh[i * n:(i + 1) * n], ph[i * n:(i + 1) * n]) == 0
+    g.close()
