@@ -768,11 +768,27 @@ __device__ __forceinline__ void bu_body(const KArgs& a, const int* kp, int* __re
     b.lvl = lvl;
     // prefill: F_{k+1} already holds look-ahead vertices of step k-1 (OR into it)
     const bool pf = LA && prefill;
+    unsigned long long oedges = 0;   // DIR: out-degrees of the found vertices, summed where they are published
     bu_chunks<WARPS, LA, XBFS_BU_H32>(b, sm, [&](long long w, unsigned vis, unsigned f, unsigned lf) {
         if (pf) f |= __ldcg(next + w);
         if (f) next[w] = f;
         a.visited[w] = vis | f | lf;
         if (LA && lf) a.la[w] = lf;
+        if constexpr (DIR) {
+            for (unsigned bits = f; bits;) {
+                unsigned long long hv[8];
+#pragma unroll
+                for (int i = 0; i < 8; ++i) {
+                    hv[i] = 0ull;
+                    if (bits) {
+                        hv[i] = __ldg(a.head + w * 32 + __ffs(bits) - 1);
+                        bits &= bits - 1;
+                    }
+                }
+#pragma unroll
+                for (int i = 0; i < 8; ++i) oedges += hv[i] >> 32;
+            }
+        }
     }, found, edges, probes, fmax, la);
     const int lane = threadIdx.x & 31;
 #pragma unroll
@@ -787,9 +803,12 @@ __device__ __forceinline__ void bu_body(const KArgs& a, const int* kp, int* __re
     }
     k = *(const volatile int*)kp;
     // directed graph: the BU rows are in-arc rows, whose lengths are not the out-degrees
-    // edgesF_{k+1} needs; the count pass (ss_count_body) that follows supplies |F_{k+1}|
-    // and edgesF_{k+1} from the out-arc head[] instead
-    if (DIR) found = edges = 0;
+    // edgesF_{k+1} needs; those were summed from the out-arc head[] at publication
+    if (DIR) {
+        edges = oedges;
+#pragma unroll
+        for (int o = 16; o; o >>= 1) edges += __shfl_xor_sync(FULL, edges, o);
+    }
     if (lane == 0 && (found | edges | probes)) {
         atomicAdd(&a.st->acc_found[k % 3], found);
         atomicAdd(&a.st->acc_edges[k % 3], edges);
@@ -1167,11 +1186,8 @@ __global__ __launch_bounds__(kPersistThreads, kPersistBlocks) void k_persist(
             grid_sync(bar, epoch);
             ss_count_body(a, k);
         } else {
+            // (directed: bu_body sums edgesF_{k+1} over out-arcs itself)
             bu_body<kPersistThreads / 32, LA, decltype(sm.bu), DIR>(a, &s.k, level, parent, sm.bu, s.prefill);
-            if constexpr (DIR) {    // |F_{k+1}|, edgesF_{k+1} over out-arcs (see bu_body)
-                grid_sync(bar, epoch);
-                ss_count_body(a, k);
-            }
         }
         grid_sync(bar, epoch);
         if (threadIdx.x == 0) select_step(a, s, blockIdx.x == 0, blockIdx.x == 0 ? globaltimer() : 0ull);

@@ -111,8 +111,8 @@ def bfs_level_bytes(n: int, strategy, fv, fe, unvisited, probes, directed: bool 
             b += bytes_td_ss(n, fv[k], fe[k], found) + bytes_ss_count(n, found)
         else:
             b += bytes_bu(n, unvisited[k], probes[k], found)
-            if directed:     # in-arc rows do not give out-degrees: the count pass follows (R-9)
-                b += bytes_ss_count(n, found)
+            if directed:     # in-arc rows do not give out-degrees: head[] of every found vertex (R-9)
+                b += 8 * found
         out.append(b)
     return out
 

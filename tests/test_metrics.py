@@ -32,15 +32,14 @@ def test_bfs_level_bytes_equals_oracle_replay():
 
 
 def test_directed_bu_level_adds_the_count_pass():
-    """R-9: a directed BU step reads in-arc rows, so |F_{k+1}| and edgesF_{k+1} come
-    from the out-arc count pass: its bytes (one bitmap + 8 B per found vertex) are
-    added to the BU level and nothing else changes."""
+    """R-9: a directed BU step reads in-arc rows, so edgesF_{k+1} comes from the
+    out-arc head[] word of every found vertex (8 B each, read where the vertex is
+    published): added to the BU level, nothing else changes."""
     from paper_conf_sc_yangls0w24_b200 import metrics
     n = 1 << 12
     strat, fv, fe, un, pr = [0, 2, 2, 0], [1, 50, 900, 30], [50, 900, 4000, 60], [4000, 3950, 3000, 2100], \
         [0, 7000, 5000, 0]
     u = metrics.bfs_level_bytes(n, strat, fv, fe, un, pr)
     d = metrics.bfs_level_bytes(n, strat, fv, fe, un, pr, directed=True)
-    B = 4 * (n // 32)
     assert d[0] == u[0] and d[3] == u[3]
-    assert d[1] - u[1] == B + 8 * 900 and d[2] - u[2] == B + 8 * 30
+    assert d[1] - u[1] == 8 * 900 and d[2] - u[2] == 8 * 30
