@@ -265,6 +265,7 @@ def run_ours(args):
     per_root = []
     launches = 0
     alg_bytes = 0
+    km_bytes = 0
     phase = {}          # strategy -> [levels, ms, algorithmic bytes] (persistent driver's level stamps)
     for r in mine:
         flush.fill_(1)                       # L2 flush, outside the timed region
@@ -272,9 +273,11 @@ def run_ours(args):
         per_root.append((int(r), st.elapsed_ms, st.input_edges_traversed, st.arcs_traversed, st.num_levels,
                          "".join("FSB"[s] for s in st.strategy)))
         launches += st.kernel_launches
-        lb = metrics.bfs_level_bytes(n, st.strategy, st.frontier_vertices, st.frontier_edges, st.unvisited,
-                                     st.bu_probes, directed=directed)
-        alg_bytes += metrics.bytes_init(n) + sum(lb)
+        lb = metrics.d3_level_bytes(n, st.strategy, st.frontier_vertices, st.frontier_edges, st.unvisited,
+                                    st.bu_probes)
+        alg_bytes += metrics.d3_init(n) + sum(lb)
+        km_bytes += metrics.kernel_model_bytes(n, st.strategy, st.frontier_vertices, st.frontier_edges,
+                                               st.unvisited, st.bu_probes, directed=directed)
         for s_, ms_, b_ in zip(st.strategy, st.level_ms, lb):
             ph = phase.setdefault("FSB"[s_], [0, 0.0, 0])
             ph[0] += 1
@@ -364,9 +367,13 @@ def run_ours(args):
                     "phases": {k: {"levels": v[0], "ms": round(v[1], 4),
                                    "gbs": round(v[2] / (v[1] * 1e-3) / 1e9, 1) if v[1] > 0 else None}
                                for k, v in phase.items()},
-                    "note": "achieved = algorithmic bytes (init + every level, DESIGN.md §5) / event time of the "
-                            "single k_persist launch per BFS, over the timed roots; phases from the kernel's "
-                            "%globaltimer level stamps"}
+                    "kernel_model": {"bytes_per_launch": int(km_bytes / len(per_root)),
+                                     "gbs": round(km_bytes / (timed_ms * 1e-3) / 1e9, 1),
+                                     "note": "what this build's kernels move by their own traffic model "
+                                             "(metrics.kernel_model_bytes); context, not the numerator"},
+                    "note": "achieved = SURVEY §8(d) D-3 algorithmic bytes (init + every level, replayed by "
+                            "oracle_byte_replay) / event time of the single k_persist launch per BFS, over the "
+                            "timed roots; phases from the kernel's %globaltimer level stamps"}
     elif agg:
         dom = max(agg.items(), key=lambda kv: kv[1][1])[0]
         d = kernels[dom]

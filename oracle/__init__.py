@@ -8,8 +8,10 @@ header and DESIGN.md §3); pins live in ``tests/test_oracle.py``.
 
 Parity status per function:
   build_csr, reorder, bfs, validate, input_edges, level_stats, select,
-  byte_replay, build_csr_directed, validate_directed — all pinned (closed
-  forms, scipy brute force, mutation tests, hand-computed replay).  The paper's own worked example (Figs 1-4) is lost:
+  select_sequence, byte_replay, build_csr_directed,
+  validate_directed, validate_tuples (OpenMP, liboracle_omp.so) — all pinned
+  (closed forms, scipy brute force, mutation tests, hand-computed replay,
+  agreement of the two validators).  The paper's own worked example (Figs 1-4) is lost:
   "parity unpinned" for that example only.
 """
 from __future__ import annotations
@@ -23,6 +25,8 @@ import numpy as np
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _SRC = os.path.join(_HERE, "oracle.c")
 _LIB = os.path.join(_HERE, "liboracle.so")
+_SRC_OMP = os.path.join(_HERE, "validate_omp.c")
+_LIB_OMP = os.path.join(_HERE, "liboracle_omp.so")
 
 V1_ROOT, V2_REACH, V3_LEVEL_STEP, V4_TREE_EDGE, V5_EDGE_SPAN, V_RANGE = 1, 2, 4, 8, 16, 32
 
@@ -31,6 +35,10 @@ def build(force: bool = False) -> str:
     """Compile oracle.c with plain gcc (no OpenMP, no CUDA)."""
     if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
         subprocess.check_call(["gcc", "-O2", "-std=c11", "-Wall", "-shared", "-fPIC", "-o", _LIB, _SRC])
+    # the tuple-list validator for s27-size roots: OpenMP over the host cores
+    if force or not os.path.exists(_LIB_OMP) or os.path.getmtime(_LIB_OMP) < os.path.getmtime(_SRC_OMP):
+        subprocess.check_call(["gcc", "-O2", "-std=c11", "-Wall", "-fopenmp", "-shared", "-fPIC", "-o", _LIB_OMP,
+                               _SRC_OMP])
     return _LIB
 
 
@@ -56,8 +64,10 @@ def lib():
         L.oracle_input_edges.restype = i64
         L.oracle_level_stats.argtypes = [i64, P, P, i32, P, P]
         L.oracle_level_stats.restype = i32
-        L.oracle_select.argtypes = [i64, i64, i64, i64, f64, f64, f64]
+        L.oracle_select.argtypes = [i64, i64, i64, i64, f64, f64, f64, f64, i32, i64]
         L.oracle_select.restype = i32
+        L.oracle_select_sequence.argtypes = [i64, P, P, i32, f64, f64, f64, f64, P, P]
+        L.oracle_select_sequence.restype = i32
         L.oracle_byte_replay.argtypes = [i64, P, P, P, i32, P, P]
         L.oracle_byte_replay.restype = i64
         L.oracle_bu_probes.argtypes = [i64, P, P, P, i32]
@@ -171,13 +181,55 @@ def level_stats(g: CSR, level):
     return fs[:nl].copy(), fe[:nl].copy()
 
 
-def select(f_size: int, f_prev: int, f_edges: int, arcs: int, alpha=0.1, grow=2.0, ratio_min=1e-3) -> int:
-    """P:L87 strategy rule (0 SF, 1 SS, 2 BU); growth rule is reading C-10."""
-    return int(lib().oracle_select(f_size, f_prev, f_edges, arcs, alpha, grow, ratio_min))
+def select(f_size: int, f_prev: int, f_edges: int, arcs: int, alpha=0.1, grow=2.0, ratio_min=1e-3,
+           bu_stay=0.0, prev=-1, unvisited=0) -> int:
+    """P:L87 strategy rule (0 SF, 1 SS, 2 BU); growth rule is reading C-10, the
+    optional stay-in-BU hysteresis (bu_stay > 0, after a BU step) reading C-11."""
+    return int(lib().oracle_select(f_size, f_prev, f_edges, arcs, alpha, grow, ratio_min, bu_stay, prev,
+                                   unvisited))
+
+
+def select_sequence(g: CSR, level, alpha=0.1, grow=2.0, ratio_min=1e-3, bu_stay=0.0):
+    """The selector replayed over one BFS (exact levels): returns (strategy int8[nl],
+    U_k int64[nl]) where U_k = non-isolated vertices unreached before step k."""
+    level = np.ascontiguousarray(level, dtype=np.int32)
+    cap = int(level.max()) + 2 if level.size else 1
+    st = np.zeros(cap, dtype=np.int8)
+    un = np.zeros(cap, dtype=np.int64)
+    nl = lib().oracle_select_sequence(g.n, _p(g.row_ptr), _p(level), cap, alpha, grow, ratio_min, bu_stay,
+                                      _p(st), _p(un))
+    if nl < 0:
+        raise ValueError("oracle_select_sequence failed")
+    return st[:nl].copy(), un[:nl].copy()
+
+
+_lib_omp = None
+
+
+def validate_tuples(n: int, src, dst, source: int, level, parent, directed: bool = False,
+                    threads: int | None = None) -> int:
+    """O-5 V1..V5 over the tuple list (no CSR), OpenMP-parallel: the s27 validator.
+    Same bitmask as validate()."""
+    global _lib_omp
+    if _lib_omp is None:
+        build()
+        L = ctypes.CDLL(_LIB_OMP)
+        P = ctypes.c_void_p
+        L.oracle_validate_tuples.argtypes = [ctypes.c_int64, ctypes.c_int64, P, P, ctypes.c_int64, P, P,
+                                             ctypes.c_int32, ctypes.c_int32]
+        L.oracle_validate_tuples.restype = ctypes.c_int
+        _lib_omp = L
+    src, dst = _u32(src), _u32(dst)
+    level = np.ascontiguousarray(level, dtype=np.int32)
+    parent = np.ascontiguousarray(parent, dtype=np.int32)
+    t = threads if threads else (os.cpu_count() or 1)
+    return _lib_omp.oracle_validate_tuples(n, src.shape[0], _p(src), _p(dst), int(source), _p(level), _p(parent),
+                                           int(bool(directed)), int(t))
 
 
 def byte_replay(g: CSR, level, strategy):
-    """O-8 algorithmic bytes of one BFS for a strategy sequence (reordered CSR)."""
+    """O-8 algorithmic bytes of one BFS for a strategy sequence (reordered CSR),
+    exactly SURVEY §8(d) D-3.  Returns (total incl. init, per-level int64[])."""
     level = np.ascontiguousarray(level, dtype=np.int32)
     strategy = np.ascontiguousarray(strategy, dtype=np.int8)
     per = np.zeros(max(len(strategy), 1), dtype=np.int64)

@@ -25,9 +25,13 @@
  *                      (the numerator of the paper's ratio).
  *   oracle_select      the paper's strategy rule (§III): BU iff
  *                      edgesF_k / |M| > alpha; otherwise SF/SS by frontier growth
- *                      (rule unstated in the paper: reading C-10).
+ *                      (rule unstated in the paper: reading C-10), plus the
+ *                      optional stay-in-BU hysteresis of reading C-11.
+ *   oracle_select_sequence  the selector replayed level by level over a BFS:
+ *                      |F_k|, edgesF_k, U_k from the level array, the rule above.
  *   oracle_byte_replay O-8: algorithmic bytes of one BFS given the per-level
- *                      strategy sequence.
+ *                      strategy sequence, exactly SURVEY §8(d) D-3 (not any
+ *                      kernel's traffic model).
  *   oracle_build_csr_directed  f4 (directed graphs; reading
  *                      R-9): out-arc CSR of the tuples taken as arcs i -> j,
  *                      self-loops and duplicate arcs dropped, rows id-sorted.
@@ -37,6 +41,9 @@
  *                      V3 as undirected; V4 the tree arc parent[v] -> v exists;
  *                      V5 for every tuple (i,j), i != j: i reached implies j
  *                      reached with level[j] <= level[i] + 1.
+ *   (validate_omp.c, liboracle_omp.so) oracle_validate_tuples: the same V1-V5
+ *                      restated over the tuple list only (no CSR), OpenMP-parallel,
+ *                      for the s27 sizes where the serial oracle is too slow.
  *
  * Parity pins: tests/test_oracle.py (closed forms, scipy brute force,
  * validator mutation tests, hand-computed byte replay).
@@ -168,6 +175,8 @@ int oracle_validate(int64_t n, const int64_t* row_ptr, const int32_t* col,
     for (int64_t v = 0; v < n; ++v) {
         int reached_l = level[v] >= 0, reached_p = parent[v] >= 0;
         if (reached_l != reached_p) { bad |= V2_REACH_CONSISTENT; continue; } /* V2 */
+        /* V2 (§8(b) semantics, reading C-1): unreached means exactly level = parent = -1 */
+        if (!reached_l && (level[v] != -1 || parent[v] != -1)) { bad |= V2_REACH_CONSISTENT; continue; }
         if (parent[v] >= n || level[v] < -1) { bad |= V_RANGE; continue; }
         if (!reached_l || v == s) continue;
         int32_t p = parent[v];
@@ -210,37 +219,81 @@ int32_t oracle_level_stats(int64_t n, const int64_t* row_ptr, const int32_t* lev
  * graph exceeds alpha, XBFS selects the bottom-up strategy.  Otherwise, it
  * switches between the scan-free and single-scan strategies based on the
  * growth rate of the number of nodes in the frontier queue."  alpha = 0.1
- * (P:L347).  Growth rule (unstated; reading C-10): single-scan iff
- * |F_k| > grow * |F_{k-1}| and ratio > ratio_min.  0 = SF, 1 = SS, 2 = BU. */
+ * (0.04 on B200, reading C-13/R-4).  Strict '>' (C-8).  Growth rule
+ * (unstated; reading C-10): single-scan iff |F_k| > grow * |F_{k-1}| and
+ * ratio > ratio_min.  Reading C-11 (optional hysteresis, bu_stay > 0): after a
+ * bottom-up step stay bottom-up while |U_k| * bu_stay < edgesF_k.
+ * prev = strategy of step k-1 (-1 at k = 0).  0 = SF, 1 = SS, 2 = BU. */
 int32_t oracle_select(int64_t f_size, int64_t f_prev, int64_t f_edges, int64_t arcs,
-                      double alpha, double grow, double ratio_min) {
+                      double alpha, double grow, double ratio_min,
+                      double bu_stay, int32_t prev, int64_t unvisited) {
     double ratio = arcs > 0 ? (double)f_edges / (double)arcs : 0.0;
     if (ratio > alpha) return 2;
+    if (bu_stay > 0.0 && prev == 2 && (double)unvisited * bu_stay < (double)f_edges) return 2;
     if ((double)f_size > grow * (double)f_prev && ratio > ratio_min) return 1;
     return 0;
 }
 
+/* The selector replayed over one BFS, in level order (P:L87 per level): from
+ * the exact level array, |F_k| = #{v : level v = k}, edgesF_k = sum of deg over
+ * F_k, U_k = non-isolated vertices not reached at levels <= k (the BU
+ * candidates of step k), and strategy[k] = oracle_select(|F_k|, |F_{k-1}|,
+ * edgesF_k, A, ..., strategy[k-1], U_k).  Arrays sized >= nlevels.
+ * Returns nlevels, or -1 if cap is too small. */
+int32_t oracle_select_sequence(int64_t n, const int64_t* row_ptr, const int32_t* level, int32_t cap,
+                               double alpha, double grow, double ratio_min, double bu_stay,
+                               int8_t* strategy, int64_t* unvisited_out) {
+    int32_t nl = 0;
+    for (int64_t v = 0; v < n; ++v) if (level[v] + 1 > nl) nl = level[v] + 1;
+    if (nl > cap) return -1;
+    int64_t* fsize = (int64_t*)calloc((size_t)nl + 1, sizeof(int64_t));
+    int64_t* fedges = (int64_t*)calloc((size_t)nl + 1, sizeof(int64_t));
+    int64_t* noniso_at = (int64_t*)calloc((size_t)nl + 1, sizeof(int64_t));
+    if (!fsize || !fedges || !noniso_at) { free(fsize); free(fedges); free(noniso_at); return -2; }
+    int64_t nonisolated = 0;
+    for (int64_t v = 0; v < n; ++v) {
+        int64_t d = row_ptr[v + 1] - row_ptr[v];
+        if (d > 0) nonisolated++;
+        if (level[v] < 0) continue;
+        fsize[level[v]]++;
+        fedges[level[v]] += d;
+        if (d > 0) noniso_at[level[v]]++;
+    }
+    const int64_t arcs = row_ptr[n];
+    int64_t reached_noniso = 0;
+    int32_t prev = -1;
+    for (int32_t k = 0; k < nl; ++k) {
+        reached_noniso += noniso_at[k];                 /* visited before step k: levels <= k */
+        int64_t u = nonisolated - reached_noniso;
+        int32_t s = oracle_select(fsize[k], k > 0 ? fsize[k - 1] : 0, fedges[k], arcs,
+                                  alpha, grow, ratio_min, bu_stay, prev, u);
+        strategy[k] = (int8_t)s;
+        if (unvisited_out) unvisited_out[k] = u;
+        prev = s;
+    }
+    free(fsize); free(fedges); free(noniso_at);
+    return nl;
+}
+
 /* ------------------------------------------------------ O-8 byte replay */
-/* Algorithmic bytes of one BFS (the per-kernel model of DESIGN.md §5), given
- * the strategy used at each level (0 SF, 1 SS, 2 BU) and the (reordered) CSR
- * the GPU traversed.  B = 4*ceil(n/32) is one n-bit bitmap pass.
- *   init        : 8n (level+parent) + 5B (visited, non-isolated, 3 frontier maps)
- *   SF step k   : B (stale frontier clear) + 20|F_k| (queue entries) + 4 edgesF_k
- *                 (col) + 44|F_{k+1}| (level 4, parent 4, row_ptr pair 16, queue 20)
- *   SS step k   : B + 20|F_k| + 4 edgesF_k + 8|F_{k+1}|, then the single scan of
- *                 the next-frontier bitmap: B + 8|F_{k+1}| (head[] degrees); the
- *                 queue is rebuilt only if the next step is top-down (below)
- *   BU step k   : 4B (visited read+write, next write, stale clear) + 16|U_k|
- *                 (row_ptr pair per candidate) + 4 probes_k (col) + 8|F_{k+1}|
- *   a TD step right after a BU or SS step first rebuilds the queue: B + 36|F_k|.
- * probes(v) = 1 + index of the first level-k neighbour in v's stored row, or
- * deg(v) if none (BU tests only level k: reading C-9).  per_level[k] gets the
+/* Algorithmic bytes of one BFS, SURVEY §8(d) D-3 exactly, given the strategy
+ * used at each level (0 SF, 1 SS, 2 BU) and the (reordered) CSR the GPU
+ * traversed.  The D-3 terms (bitmap probes are L2 traffic, not counted):
+ *   init       : 8N (level + parent) + 3N/8 (three N-bit bitmaps)
+ *   TD step k  : 20|F_k| (queue entry + row_ptr pair) + 4 edgesF_k (col)
+ *                + 28|F_{k+1}| (level 4, parent 4, queue 4, row_ptr pair 16 for binning)
+ *   SS step k  : the TD terms + N/8 (single-scan generation over the N-bit status bitmap)
+ *   BU step k  : N/4 (two bitmaps) + 24|U_k| + 4 probes_k (col) + 8|F_{k+1}| (level, parent)
+ * N/8 is rounded up to whole bytes (reading R-11): bm = ceil(N/8), N/4 = 2 bm,
+ * 3N/8 = 3 bm.  probes(v) = 1 + index of the first level-k neighbour in v's
+ * stored row, or deg(v) if none (BU tests only level k: reading C-9); U_k =
+ * non-isolated vertices not reached at levels <= k.  per_level[k] gets the
  * bytes of step k; the return value includes init. */
 int64_t oracle_byte_replay(int64_t n, const int64_t* row_ptr, const int32_t* col,
                            const int32_t* level, int32_t nlevels, const int8_t* strategy,
                            int64_t* per_level) {
-    const int64_t B = 4 * ((n + 31) / 32);
-    int64_t total = 8 * n + 5 * B;
+    const int64_t bm = (n + 7) / 8;
+    int64_t total = 8 * n + 3 * bm;
     int64_t* fsize = (int64_t*)calloc((size_t)nlevels + 1, sizeof(int64_t));
     int64_t* fedges = (int64_t*)calloc((size_t)nlevels + 1, sizeof(int64_t));
     if (!fsize || !fedges) { free(fsize); free(fedges); return -1; }
@@ -253,7 +306,6 @@ int64_t oracle_byte_replay(int64_t n, const int64_t* row_ptr, const int32_t* col
     int64_t unvisited = nonisolated;     /* U_0: non-isolated vertices other than the source */
     for (int64_t v = 0; v < n; ++v)
         if (level[v] == 0 && row_ptr[v + 1] > row_ptr[v]) unvisited--;
-    int prev_bu = 0;
     for (int32_t k = 0; k < nlevels; ++k) {
         int64_t bytes = 0;
         int64_t found = fsize[k + 1];                        /* |F_{k+1}| (0 past the end) */
@@ -267,13 +319,10 @@ int64_t oracle_byte_replay(int64_t n, const int64_t* row_ptr, const int32_t* col
                     if (level[col[p]] == k) { pr = p - row_ptr[v] + 1; break; }
                 probes += pr;
             }
-            bytes = 4 * B + 16 * unvisited + 4 * probes + 8 * found;
-            prev_bu = 1;
+            bytes = 2 * bm + 24 * unvisited + 4 * probes + 8 * found;
         } else {
-            if (prev_bu) bytes += B + 36 * fsize[k];            /* queue rebuilt from the bitmap */
-            bytes += B + 20 * fsize[k] + 4 * fedges[k];
-            if (strategy[k] == 0) { bytes += 44 * found; prev_bu = 0; }
-            else { bytes += 8 * found + B + 8 * found; prev_bu = 1; }   /* single scan, no queue */
+            bytes = 20 * fsize[k] + 4 * fedges[k] + 28 * found;
+            if (strategy[k] == 1) bytes += bm;                  /* SS: the single scan */
         }
         unvisited -= found;
         if (per_level) per_level[k] = bytes;
@@ -360,6 +409,8 @@ int oracle_validate_directed(int64_t n, const int64_t* row_ptr, const int32_t* c
     for (int64_t v = 0; v < n; ++v) {
         int reached_l = level[v] >= 0, reached_p = parent[v] >= 0;
         if (reached_l != reached_p) { bad |= V2_REACH_CONSISTENT; continue; } /* V2 */
+        /* V2 (§8(b) semantics, reading C-1): unreached means exactly level = parent = -1 */
+        if (!reached_l && (level[v] != -1 || parent[v] != -1)) { bad |= V2_REACH_CONSISTENT; continue; }
         if (parent[v] >= n || level[v] < -1) { bad |= V_RANGE; continue; }
         if (!reached_l || v == s) continue;
         int32_t p = parent[v];

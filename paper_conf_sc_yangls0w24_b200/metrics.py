@@ -46,10 +46,46 @@ def quartiles(xs: Sequence[float]):
 
 
 # --------------------------------------------------------------------------
-# Algorithmic bytes per kernel launch.  Inputs are the per-level
-# counters the library logs; used for the bench's live roofline figure.
-# B = 4*ceil(n/32) bytes is one pass over an n-bit bitmap.  Bitmap probes per
-# arc are L2 traffic (the bitmaps are L2-resident) and are not counted.
+# the ALGORITHMIC bytes of one BFS given the strategies the
+# selector took (the roofline numerator; replayed independently by the oracle's
+# oracle_byte_replay, tests/test_metrics.py).  Bitmap probes are L2 traffic and
+# are not counted.  N/8 is rounded up to whole bytes (reading R-11).
+# --------------------------------------------------------------------------
+
+def d3_bitmap(n: int) -> int:
+    """N/8 bytes (one N-bit bitmap), rounded up."""
+    return (n + 7) // 8
+
+
+def d3_init(n: int) -> int:
+    """level + parent (8N) + three N-bit bitmaps (3N/8)."""
+    return 8 * n + 3 * d3_bitmap(n)
+
+
+def d3_level_bytes(n: int, strategy, fv, fe, unvisited, probes):
+    """Per level k: TD (SF/SS) 20|F_k| + 4 edgesF_k + 28|F_{k+1}| (+ N/8 for the
+    single scan of SS); BU N/4 + 24|U_k| + 4 probes_k + 8|F_{k+1}|."""
+    bm = d3_bitmap(n)
+    out = []
+    L = len(strategy)
+    for k in range(L):
+        found = fv[k + 1] if k + 1 < L else 0
+        if strategy[k] == 2:
+            out.append(2 * bm + 24 * unvisited[k] + 4 * probes[k] + 8 * found)
+        else:
+            out.append(20 * fv[k] + 4 * fe[k] + 28 * found + (bm if strategy[k] == 1 else 0))
+    return out
+
+
+def d3_bytes(n: int, strategy, fv, fe, unvisited, probes) -> int:
+    """Init + every level: D-3 algorithmic bytes of one whole BFS."""
+    return d3_init(n) + sum(d3_level_bytes(n, strategy, fv, fe, unvisited, probes))
+
+
+# --------------------------------------------------------------------------
+# KERNEL TRAFFIC MODEL (reported as the bench line's `kernel_model`, never as
+# the roofline numerator): what this build's kernels move per launch
+# (DESIGN.md §5).  B = 4*ceil(n/32) bytes is one pass over an n-bit bitmap.
 # --------------------------------------------------------------------------
 
 def bitmap_bytes(n: int) -> int:
@@ -91,7 +127,7 @@ def bytes_ss_count(n: int, found: int) -> int:
     return bitmap_bytes(n) + 8 * found
 
 
-def bfs_level_bytes(n: int, strategy, fv, fe, unvisited, probes, directed: bool = False):
+def kernel_model_level_bytes(n: int, strategy, fv, fe, unvisited, probes, directed: bool = False):
     """Algorithmic bytes of every level of one BFS given the strategies the
     selector took (the phases of the persistent kernel): SF and SS
     read a queue that exists after an SF level (No-Frontier-Generation) and is
@@ -117,6 +153,6 @@ def bfs_level_bytes(n: int, strategy, fv, fe, unvisited, probes, directed: bool 
     return out
 
 
-def bfs_alg_bytes(n: int, strategy, fv, fe, unvisited, probes, directed: bool = False) -> int:
+def kernel_model_bytes(n: int, strategy, fv, fe, unvisited, probes, directed: bool = False) -> int:
     """Init + every level: the algorithmic bytes of one persistent-kernel launch."""
-    return bytes_init(n) + sum(bfs_level_bytes(n, strategy, fv, fe, unvisited, probes, directed))
+    return bytes_init(n) + sum(kernel_model_level_bytes(n, strategy, fv, fe, unvisited, probes, directed))

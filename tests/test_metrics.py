@@ -1,19 +1,20 @@
-"""Harness arithmetic against the oracle: the bench's per-BFS algorithmic byte
-count (metrics.bfs_level_bytes, the persistent kernel's roofline numerator)
-equals the oracle's byte replay (O-8, itself pinned by hand in test_oracle.py)
-for any strategy sequence."""
+"""Harness arithmetic against the oracle: the bench's roofline numerator
+(metrics.d3_level_bytes / d3_bytes) equals the oracle's byte
+replay (O-8, itself pinned by hand in test_oracle.py) for any strategy
+sequence, given the per-level counters the library logs."""
 import numpy as np
 
 import oracle
 from paper_conf_sc_yangls0w24_b200 import metrics, synth
 
 
-def test_bfs_level_bytes_equals_oracle_replay():
+def test_d3_bytes_equal_oracle_replay():
     src, dst, n = synth.kronecker(11, seed=3)
+    n = n + 5                                   # N not a multiple of 8 (R-11 rounding) + isolated tail
     g = oracle.reorder(oracle.build_csr(n, src, dst))
     rng = np.random.default_rng(0)
     nonisolated = int((np.diff(g.row_ptr) > 0).sum())
-    for root in synth.roots(n, src, dst, 3, root_seed=4):
+    for root in synth.roots(n - 5, src, dst, 3, root_seed=4):
         level, _, nl = oracle.bfs(g, int(root))
         fs, fe = oracle.level_stats(g, level)
         for _ in range(6):
@@ -25,21 +26,16 @@ def test_bfs_level_bytes_equals_oracle_replay():
                 unv.append(u)
                 probes.append(oracle.bu_probes(g, level, k) if strat[k] == 2 else 0)
                 u -= int(fs[k + 1]) if k + 1 < nl else 0
-            mine = metrics.bfs_level_bytes(n, strat, fs.tolist(), fe.tolist(), unv, probes)
+            mine = metrics.d3_level_bytes(n, strat, fs.tolist(), fe.tolist(), unv, probes)
             assert mine == per.tolist()
-            assert metrics.bfs_alg_bytes(n, strat, fs.tolist(), fe.tolist(), unv, probes) == \
+            assert metrics.d3_bytes(n, strat, fs.tolist(), fe.tolist(), unv, probes) == \
                 oracle.byte_replay(g, level, strat)[0]
 
 
-def test_directed_bu_level_adds_the_count_pass():
-    """R-9: a directed BU step reads in-arc rows, so edgesF_{k+1} comes from the
-    out-arc head[] word of every found vertex (8 B each, read where the vertex is
-    published): added to the BU level, nothing else changes."""
-    from paper_conf_sc_yangls0w24_b200 import metrics
+def test_d3_terms_by_hand():
+    """D-3 at N = 4096 (N/8 = 512): init 8N + 3N/8; an SF, an SS and a BU level."""
     n = 1 << 12
-    strat, fv, fe, un, pr = [0, 2, 2, 0], [1, 50, 900, 30], [50, 900, 4000, 60], [4000, 3950, 3000, 2100], \
-        [0, 7000, 5000, 0]
-    u = metrics.bfs_level_bytes(n, strat, fv, fe, un, pr)
-    d = metrics.bfs_level_bytes(n, strat, fv, fe, un, pr, directed=True)
-    assert d[0] == u[0] and d[3] == u[3]
-    assert d[1] - u[1] == 8 * 900 and d[2] - u[2] == 8 * 30
+    strat, fv, fe, un, pr = [0, 1, 2], [1, 50, 900], [50, 900, 4000], [4000, 3950, 3000], [0, 0, 5000]
+    assert metrics.d3_init(n) == 8 * 4096 + 3 * 512
+    lv = metrics.d3_level_bytes(n, strat, fv, fe, un, pr)
+    assert lv == [20 * 1 + 4 * 50 + 28 * 50, 20 * 50 + 4 * 900 + 28 * 900 + 512, 1024 + 24 * 3000 + 4 * 5000]

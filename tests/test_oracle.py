@@ -210,8 +210,8 @@ def test_reorder_invariants():
 
 def _valid_case():
     rng = np.random.default_rng(11)
-    n = 200
-    e = rng.integers(0, n, (800, 2))
+    n = 220                                   # vertices 200..219 are isolated (never reached)
+    e = rng.integers(0, 200, (800, 2))
     n, src, dst = _graph(n, e)
     g = oracle.build_csr(n, src, dst)
     s = int(src[0])
@@ -256,9 +256,14 @@ def test_validator_rejects_mutations():
 
     # an unreached vertex marked reached with a bogus parent
     un = np.flatnonzero(level == -1)
-    if un.size:
-        lv = level.copy(); p = parent.copy(); lv[un[0]] = 1; p[un[0]] = s
-        assert oracle.validate(g, src, dst, s, lv, p) != 0
+    assert un.size
+    lv = level.copy(); p = parent.copy(); lv[un[0]] = 1; p[un[0]] = s
+    assert oracle.validate(g, src, dst, s, lv, p) != 0
+
+    # §8(b): an unreached vertex holds exactly level = parent = -1 (any other negative fails)
+    for bad_l, bad_p in ((-1, -2), (-7, -1), (-7, -7), (-1, -2147483648)):
+        lv = level.copy(); p = parent.copy(); lv[un[0]] = bad_l; p[un[0]] = bad_p
+        assert oracle.validate(g, src, dst, s, lv, p) & oracle.V2_REACH, (bad_l, bad_p)
 
 
 # ----------------------------------------------------------- TEPS / stats pins
@@ -310,29 +315,82 @@ def test_selector_paper_rule_on_table3():
 
 
 def test_byte_replay_hand_computed():
-    """Path 0-1-2-3 from s=0 (n=4, one bitmap word: B = 4 bytes), strategies
-    SF, BU, SF, SF.  deg = [1,2,2,1]; F = {0},{1},{2},{3}.
-      init      8*4 + 5*4                                        = 52
-      L0 SF     B + 20*|F0| + 4*edgesF0(1) + 44*|F1|              = 4+20+4+44   = 72
-      L1 BU     4B + 16*U1 + 4*probes + 8*|F2|, U1 = {2,3}
+    """SURVEY §8(d) D-3 by hand.  Path 0-1-2-3 from s=0 (N=4: N/8 -> bm = 1 byte,
+    reading R-11), strategies SF, BU, SF, SF.  deg = [1,2,2,1]; F = {0},{1},{2},{3}.
+      init      8N + 3N/8                                  = 32 + 3         = 35
+      L0 SF     20|F0| + 4 edgesF0 + 28|F1|                = 20 + 4 + 28    = 52
+      L1 BU     N/4 + 24|U1| + 4 probes + 8|F2|, U1 = {2,3}
                 probes: v2's reordered row [1 (deg 2), 3 (deg 1)] -> 1
                         v3's row [2]: no level-1 neighbour -> deg 1  => 2
-                                                                  = 16+32+8+8   = 64
-      L2 SF     rebuild queue after BU: B + 36*|F2| = 40; then
-                B + 20 + 4*edgesF2(2) + 44*|F3|                   = 40+4+20+8+44 = 116
-      L3 SF     B + 20 + 4*1 + 0                                  = 28
-    SS variant at L2: 40 + (4 + 20 + 8 + 8*1) + (4 + 8*1)         = 92
-    and the SF step after it rebuilds the queue again: 40 + 28    = 68
+                                                           = 2 + 48 + 8 + 8 = 66
+      L2 SF     20 + 4*2 + 28                                               = 56
+      L3 SF     20 + 4*1 + 0                                                = 24
+    SS at L2 adds the single scan N/8: 57; D-3 charges no queue rebuild after BU.
     """
     n, src, dst = _graph(4, [(0, 1), (1, 2), (2, 3)])
     g = oracle.reorder(oracle.build_csr(n, src, dst))
     level, _, nl = oracle.bfs(g, 0)
     assert nl == 4
     tot, per = oracle.byte_replay(g, level, [0, 2, 0, 0])
-    assert per.tolist() == [72, 64, 116, 28]
-    assert tot == 52 + 72 + 64 + 116 + 28
+    assert per.tolist() == [52, 66, 56, 24]
+    assert tot == 35 + 52 + 66 + 56 + 24
     _, per2 = oracle.byte_replay(g, level, [0, 2, 1, 0])
-    assert per2[2] == 92 and per2[3] == 68
+    assert per2.tolist() == [52, 66, 57, 24]
+
+
+def test_byte_replay_hand_computed_star_rounding():
+    """Star, centre 0 with leaves 1..19 (N = 20: bm = ceil(20/8) = 3 bytes), from
+    s = 1, strategies SF, BU, SF.  F = {1}, {0}, {2..19}.
+      init   8*20 + 3*3                                  = 169
+      L0 SF  20*1 + 4*1 + 28*1                           = 52
+      L1 BU  U1 = 18 leaves, each row [0] hits at once (18 probes), 18 found:
+             2*3 + 24*18 + 4*18 + 8*18                   = 654
+      L2 SF  20*18 + 4*18 + 0                            = 432
+    All-BU instead: L0 BU: U0 = 19 (every vertex but the source), probes: v0's row
+    [1, ...] hits at index 0 -> 1, 18 leaves scan their whole row [0] -> 18 => 19;
+      2*3 + 24*19 + 4*19 + 8*1 = 546."""
+    n, src, dst = _graph(20, [(0, i) for i in range(1, 20)])
+    g = oracle.reorder(oracle.build_csr(n, src, dst))
+    level, _, nl = oracle.bfs(g, 1)
+    assert nl == 3
+    tot, per = oracle.byte_replay(g, level, [0, 2, 0])
+    assert per.tolist() == [52, 654, 432] and tot == 169 + 52 + 654 + 432
+    _, per_bu = oracle.byte_replay(g, level, [2, 2, 2])
+    assert per_bu[0] == 546
+
+
+def test_select_hysteresis_and_sequence_hand_computed():
+    """Reading C-11: after a BU step stay BU while |U_k| * bu_stay < edgesF_k;
+    never from a top-down step.  Sequence replay by hand on the star of the
+    previous test (A = 38 arcs) from s = 1, alpha = 0.1:
+      k=0: |F|=1, edgesF=1  (ratio 0.026)  -> growth 1 > 2*0 and ratio > 1e-3: SS
+      k=1: |F|=1, edgesF=19 (ratio 0.5)    -> BU
+      k=2: |F|=18, edgesF=18 (ratio 0.47)  -> BU;  U = [19, 18, 0]."""
+    assert oracle.select(10, 10, 50, 100000, alpha=0.1, bu_stay=1.0, prev=2, unvisited=49) == 2
+    assert oracle.select(10, 10, 50, 100000, alpha=0.1, bu_stay=1.0, prev=2, unvisited=50) == 0
+    assert oracle.select(10, 10, 50, 100000, alpha=0.1, bu_stay=1.0, prev=0, unvisited=1) == 0
+    assert oracle.select(10, 10, 50, 100000, alpha=0.1, bu_stay=0.0, prev=2, unvisited=1) == 0
+    n, src, dst = _graph(20, [(0, i) for i in range(1, 20)])
+    g = oracle.build_csr(n, src, dst)
+    level, _, _ = oracle.bfs(g, 1)
+    st, un = oracle.select_sequence(g, level, alpha=0.1, grow=2.0, ratio_min=1e-3, bu_stay=1.0)
+    assert st.tolist() == [1, 2, 2] and un.tolist() == [19, 18, 0]
+    # path 0..9 from 0 (A = 18): edgesF_k = 1 at k = 0 and 9, 2 elsewhere; BU iff
+    # edgesF_k / 18 > 0.1; level 0 grows (1 > 2*0) -> SS, level 9 does not -> SF
+    n, src, dst = _graph(10, [(i, i + 1) for i in range(9)])
+    g = oracle.build_csr(n, src, dst)
+    level, _, _ = oracle.bfs(g, 0)
+    st, un = oracle.select_sequence(g, level, alpha=0.1, grow=2.0, ratio_min=1e-3, bu_stay=0.0)
+    assert st.tolist() == [1, 2, 2, 2, 2, 2, 2, 2, 2, 0]
+    # every step equals the single-step rule on the exact per-level counters
+    fs, fe = oracle.level_stats(g, level)
+    prev = -1
+    for k in range(len(st)):
+        expect = oracle.select(int(fs[k]), int(fs[k - 1]) if k else 0, int(fe[k]), g.arcs, alpha=0.1, grow=2.0,
+                               ratio_min=1e-3, bu_stay=0.0, prev=prev, unvisited=int(un[k]))
+        assert st[k] == expect
+        prev = expect
+    assert un.tolist() == [9 - k for k in range(10)]
 
 
 # ------------------------------------------------------- paper byte model pin
@@ -475,9 +533,69 @@ def test_directed_validator_rejects_mutations():
     lv = level.copy(); p = parent.copy(); lv[j] = -1; p[j] = -1
     if j != s:
         assert oracle.validate_directed(g, src, dst, s, lv, p) & oracle.V5_EDGE_SPAN
+    # an unreached vertex holds exactly level = parent = -1
+    un = np.flatnonzero(level == -1)
+    assert un.size
+    for bad_l, bad_p in ((-1, -2), (-7, -7)):
+        lv = level.copy(); p = parent.copy(); lv[un[0]] = bad_l; p[un[0]] = bad_p
+        assert oracle.validate_directed(g, src, dst, s, lv, p) & oracle.V2_REACH
     # the undirected validator would reject a valid directed tree of a one-way path
     n2, s2, d2 = _graph(3, [(0, 1), (1, 2)])
     g2 = oracle.build_csr_directed(n2, s2, d2)
     lv2, pa2, _ = oracle.bfs(g2, 1)
     assert oracle.validate_directed(g2, s2, d2, 1, lv2, pa2) == 0
     assert oracle.validate(oracle.build_csr(n2, s2, d2), s2, d2, 1, lv2, pa2) & oracle.V5_EDGE_SPAN
+
+
+# ------------------------------------- O-5 over the tuple list (s27 validator)
+
+def _mutations(g, src, dst, s, level, parent):
+    """(level, parent) variants: the valid tree plus one mutation per V-check."""
+    out = [(level, parent)]
+    reached = np.flatnonzero(level >= 2)
+    v = int(reached[0])
+    p = parent.copy(); p[s] = int(reached[1]); out.append((level, p))
+    same = [u for u in np.flatnonzero(level == level[v] - 1)
+            if not np.isin(v, g.col[g.row_ptr[u]:g.row_ptr[u + 1]])]
+    p = parent.copy(); p[v] = int(same[0]); out.append((level, p))
+    u = int(parent[v]); p = parent.copy(); p[u] = v; out.append((level, p))
+    lv = level.copy(); lv[v] = -1; out.append((lv, parent))
+    lv = level.copy(); lv[level >= 2] += 1; out.append((lv, parent))
+    un = np.flatnonzero(level == -1)
+    lv = level.copy(); p = parent.copy(); lv[un[0]] = 1; p[un[0]] = s; out.append((lv, p))
+    lv = level.copy(); p = parent.copy(); p[un[0]] = -2; out.append((lv, p))
+    lv = level.copy(); p = parent.copy(); lv[un[0]] = -7; p[un[0]] = -7; out.append((lv, p))
+    lv = level.copy(); lv[s] = 1; out.append((lv, parent))
+    return out
+
+
+def test_validate_tuples_agrees_with_csr_validator():
+    """The OpenMP tuple-list validator (oracle_validate_tuples) is pinned to the
+    CSR validator: same bitmask on the valid tree and on every mutation, and zero
+    exactly when the CSR validator says valid; 1 and 4 threads agree."""
+    g, src, dst, s, level, parent = _valid_case()
+    for lv, pa in _mutations(g, src, dst, s, level, parent):
+        want = oracle.validate(g, src, dst, s, lv, pa)
+        for t in (1, 4):
+            got = oracle.validate_tuples(g.n, src, dst, s, lv, pa, threads=t)
+            assert got == want, (got, want)
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_validate_tuples_random_graphs(seed):
+    rng = np.random.default_rng(900 + seed)
+    n = int(rng.integers(2, 300))
+    e = rng.integers(0, n, (int(rng.integers(1, 4 * n)), 2))
+    n, src, dst = _graph(n, e)
+    g = oracle.build_csr(n, src, dst)
+    gd = oracle.build_csr_directed(n, src, dst)
+    for s in rng.integers(0, n, 4):
+        lv, pa, _ = oracle.bfs(g, int(s))
+        assert oracle.validate_tuples(n, src, dst, int(s), lv, pa) == 0
+        lvd, pad, _ = oracle.bfs(gd, int(s))
+        assert oracle.validate_tuples(n, src, dst, int(s), lvd, pad, directed=True) == 0
+        # the undirected tree is not a valid directed one unless the arcs allow it, and vice versa
+        assert (oracle.validate_tuples(n, src, dst, int(s), lvd, pad) == 0) == \
+            (oracle.validate(g, src, dst, int(s), lvd, pad) == 0)
+        assert (oracle.validate_tuples(n, src, dst, int(s), lv, pa, directed=True) == 0) == \
+            (oracle.validate_directed(gd, src, dst, int(s), lv, pa) == 0)
