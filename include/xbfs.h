@@ -106,7 +106,7 @@ typedef struct {
     /* Per-launch timing (measurement only): when kernel_capacity > 0 the host-loop
      * driver brackets every kernel with CUDA events on the handle's stream and
      * fills up to kernel_capacity entries (caller-owned host arrays). */
-    int32_t kernel_capacity;
+    int32_t kernel_capacity;       /* at most 4096 launches are recorded (event pool made at build time) */
     int32_t num_kernels;           /* launches recorded */
     int32_t* kernel_id;            /* XBFS_K_* */
     int32_t* kernel_level;         /* level k the launch belongs to (-1 = init) */
@@ -116,6 +116,9 @@ typedef struct {
     float* level_ms;
     /* [level_capacity] vertices step k set to level k+2 through the BU look-ahead (0 if off) */
     int64_t* lookahead_found;
+    /* persistent driver: device time (%globaltimer) from the kernel's first CTA entry to the end of
+     * the per-BFS init + seed phase; 0 under the other drivers */
+    float init_ms;
 } xbfs_run_stats;
 
 /* kernel ids reported in xbfs_run_stats.kernel_id */

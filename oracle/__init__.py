@@ -56,6 +56,10 @@ def lib():
         L.oracle_build_csr.restype = ctypes.c_int
         L.oracle_reorder.argtypes = [i64, P, P]
         L.oracle_reorder.restype = ctypes.c_int
+        L.oracle_reorder_by.argtypes = [i64, P, P, P]
+        L.oracle_reorder_by.restype = ctypes.c_int
+        L.oracle_first_parents.argtypes = [i64, P, P, P, i64, P]
+        L.oracle_first_parents.restype = i64
         L.oracle_bfs.argtypes = [i64, P, P, i64, P, P]
         L.oracle_bfs.restype = i32
         L.oracle_validate.argtypes = [i64, P, P, i64, P, P, i64, P, P]
@@ -136,13 +140,33 @@ def validate_directed(g: CSR, src, dst, source: int, level, parent) -> int:
                                           int(source), _p(level), _p(parent))
 
 
-def reorder(g: CSR) -> CSR:
-    """a2: per-row degree-descending, id-ascending ties (C-12)."""
+def reorder(g: CSR, deg_from: CSR | None = None) -> CSR:
+    """a2: per-row degree-descending, id-ascending ties (C-12).  deg_from:
+    take the neighbour degrees from this CSR instead (directed in-arc rows by the
+    in-neighbour's out-degree, R-9)."""
     col = g.col.copy()
-    rc = lib().oracle_reorder(g.n, _p(g.row_ptr), _p(col))
+    if deg_from is None:
+        rc = lib().oracle_reorder(g.n, _p(g.row_ptr), _p(col))
+    else:
+        rc = lib().oracle_reorder_by(g.n, _p(g.row_ptr), _p(col), _p(deg_from.row_ptr))
     if rc != 0:
         raise ValueError("oracle_reorder failed")
     return CSR(g.n, g.row_ptr, col)
+
+
+def transpose_directed(n: int, src, dst) -> CSR:
+    """In-arc CSR of the directed tuple graph: row j lists every i with an arc i -> j."""
+    return build_csr_directed(n, dst, src)
+
+
+def first_parents(rows: CSR, level, source: int):
+    """Reading R-12: parent[v] = first vertex of v's stored row at level[v] - 1
+    (rows = the re-arranged CSR the GPU searches).  Returns (parent int32[n], orphans)."""
+    level = np.ascontiguousarray(level, dtype=np.int32)
+    parent = np.empty(rows.n, dtype=np.int32)
+    orphans = lib().oracle_first_parents(rows.n, _p(rows.row_ptr), _p(rows.col), _p(level), int(source),
+                                         _p(parent))
+    return parent, int(orphans)
 
 
 def bfs(g: CSR, source: int):

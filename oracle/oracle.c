@@ -15,6 +15,11 @@
  *   oracle_reorder     a2: degree-aware neighbour re-arrangement (P:L153
  *                      §IV-B): each row sorted by neighbour degree descending,
  *                      ties by id ascending (reading C-12).
+ *   oracle_reorder_by  the same with degrees from another CSR (directed in-arc
+ *                      rows ordered by the in-neighbour's out-degree, R-9).
+ *   oracle_first_parents  reading R-12: parent[v] = the first vertex of v's
+ *                      stored row one level up (the CUDA path's deterministic
+ *                      choice among the valid parents of C-14).
  *   oracle_bfs         O-4: textbook FIFO-queue BFS; the "status array" holds
  *                      the visit level, level[s] = 0 (C-6), -1 = not
  *                      reached (C-1), parent[s] = s.
@@ -113,13 +118,20 @@ static int cmp_deg_desc(const void* a, const void* b) {
     return (x > y) - (x < y);                 /* tie: id ascending (C-12) */
 }
 
-int oracle_reorder(int64_t n, const int64_t* row_ptr, int32_t* col) {
-    if (n <= 0 || !row_ptr || !col) return 1;
-    g_rp = row_ptr;
+/* Rows of (row_ptr, col) sorted by the neighbour's degree in deg_row_ptr's CSR,
+ * descending, ties id ascending.  Undirected: deg_row_ptr = row_ptr.  Directed
+ * (R-9): the in-arc rows are ordered by the in-neighbour's OUT-degree. */
+int oracle_reorder_by(int64_t n, const int64_t* row_ptr, int32_t* col, const int64_t* deg_row_ptr) {
+    if (n <= 0 || !row_ptr || !col || !deg_row_ptr) return 1;
+    g_rp = deg_row_ptr;
     for (int64_t v = 0; v < n; ++v)
         qsort(col + row_ptr[v], (size_t)(row_ptr[v + 1] - row_ptr[v]), sizeof(int32_t), cmp_deg_desc);
     g_rp = NULL;
     return 0;
+}
+
+int oracle_reorder(int64_t n, const int64_t* row_ptr, int32_t* col) {
+    return oracle_reorder_by(n, row_ptr, col, row_ptr);
 }
 
 /* ------------------------------------------------------------- O-4 BFS */
@@ -148,6 +160,25 @@ int32_t oracle_bfs(int64_t n, const int64_t* row_ptr, const int32_t* col, int64_
     }
     free(Q);
     return maxl + 1;
+}
+
+/* Reading R-12 (C-14 "any valid parent", made deterministic): parent[s] = s;
+ * for every other reached v, the FIRST u in v's stored row (row_ptr/col as
+ * given: the re-arranged rows; the in-arc rows of a directed graph)
+ * with level[u] == level[v] - 1; -1 if unreached.  Returns the number of
+ * reached v != s without such a neighbour (0 for a true BFS level array). */
+int64_t oracle_first_parents(int64_t n, const int64_t* row_ptr, const int32_t* col, const int32_t* level,
+                             int64_t s, int32_t* parent) {
+    int64_t orphans = 0;
+    for (int64_t v = 0; v < n; ++v) {
+        parent[v] = -1;
+        if (level[v] < 0) continue;
+        if (v == s) { parent[v] = (int32_t)s; continue; }
+        for (int64_t p = row_ptr[v]; p < row_ptr[v + 1]; ++p)
+            if (level[col[p]] == level[v] - 1) { parent[v] = col[p]; break; }
+        if (parent[v] < 0) orphans++;
+    }
+    return orphans;
 }
 
 /* ------------------------------------------------- O-5 Graph500 checks */

@@ -118,7 +118,7 @@ void xbfs_destroy(xbfs_graph* g) {
     cudaSetDevice(g->device);
     if (g->stream) cudaStreamSynchronize(g->stream);
     if (g->copy_stream) cudaStreamSynchronize(g->copy_stream);
-    g->drop_loops();
+    if (g->loop_exec) cudaGraphExecDestroy(g->loop_exec);
     void* dev[] = {g->row_ptr, g->col, g->tcount, g->nonisolated, g->visited, g->fb, g->qv,
                    g->qoff, g->qdelta, g->tile_first, g->st, g->log, g->red_scratch,
                    g->scratch_level, g->scratch_parent, g->head, g->head32,

@@ -234,10 +234,9 @@ __device__ __forceinline__ void init_body(const KArgs& a, int* __restrict__ leve
     }
 }
 
-__global__ __launch_bounds__(256) void k_init_fill(KArgs a, int* __restrict__ level, int* __restrict__ parent,
-                                                   const unsigned int* __restrict__ nonisolated) {
+__global__ __launch_bounds__(256) void k_init_fill(KArgs a, const unsigned int* __restrict__ nonisolated) {
     count_launch(a.st);
-    init_body(a, level, parent, nonisolated);
+    init_body(a, a.st->out_level, a.st->out_parent, nonisolated);
 }
 
 __device__ int choose_strategy(const DevState* st, long long arcs, long long fsize, long long fprev,
@@ -303,10 +302,9 @@ __device__ __forceinline__ void seed_body(const KArgs& a, int* level, int* paren
     st->strategy = choose_strategy(st, a.arcs, 1, 0, deg, st->unvisited, -1);
 }
 
-__global__ void k_seed(KArgs a, int* level, int* parent, long long nonisolated_count,
-                       const unsigned int* __restrict__ nonisolated) {
+__global__ void k_seed(KArgs a, long long nonisolated_count, const unsigned int* __restrict__ nonisolated) {
     count_launch(a.st);
-    seed_body(a, level, parent, nonisolated_count, nonisolated, false);
+    seed_body(a, a.st->out_level, a.st->out_parent, nonisolated_count, nonisolated, false);
     mirror_host(a, a.st);
 }
 
@@ -605,11 +603,10 @@ __device__ __forceinline__ void td_expand_body(const KArgs& a, int k, int* __res
 }
 
 template <int MODE>
-__global__ __launch_bounds__(kExpandThreads, 3) void k_td_expand(KArgs a, int* __restrict__ level,
-                                                                int* __restrict__ parent) {
+__global__ __launch_bounds__(kExpandThreads, 2) void k_td_expand(KArgs a) {
     count_launch(a.st);
     __shared__ TdSmem sm;
-    td_expand_body<MODE, kExpandThreads>(a, a.st->k, level, parent, sm);
+    td_expand_body<MODE, kExpandThreads>(a, a.st->k, a.st->out_level, a.st->out_parent, sm);
 }
 
 // -------------------------------------------------------------- generate
@@ -839,11 +836,10 @@ __device__ __forceinline__ void la_merge(const KArgs& a, int knext) {
     }
 }
 
-__global__ __launch_bounds__(kBuThreads, 4) void k_bu_traverse(KArgs a, int* __restrict__ level,
-                                                            int* __restrict__ parent) {
+__global__ __launch_bounds__(kBuThreads, 4) void k_bu_traverse(KArgs a) {
     count_launch(a.st);
     __shared__ BuSmem<kBuThreads / 32> sm;
-    bu_body<kBuThreads / 32, false>(a, &a.st->k, level, parent, sm, false);
+    bu_body<kBuThreads / 32, false>(a, &a.st->k, a.st->out_level, a.st->out_parent, sm, false);
 }
 
 // ---------------------------------------------------------------- select
@@ -898,9 +894,10 @@ __device__ __forceinline__ bool sf_claim(unsigned int* visited, int v) {
     return !(atomicOr(visited + (v >> 5), bit) & bit);
 }
 
-__global__ void __cluster_dims__(kSmallCluster, 1, 1) __launch_bounds__(kSmallThreads, 1) k_small_sf(KArgs a, int* __restrict__ level,
-                                                             int* __restrict__ parent) {
+__global__ void __cluster_dims__(kSmallCluster, 1, 1) __launch_bounds__(kSmallThreads, 1) k_small_sf(KArgs a) {
     count_launch(a.st);
+    int* __restrict__ level = a.st->out_level;
+    int* __restrict__ parent = a.st->out_parent;
     cg::cluster_group cl = cg::this_cluster();
     const int crank = (int)cl.block_rank(), csize = (int)cl.num_blocks();
     DevState* st = a.st;
@@ -1143,13 +1140,15 @@ union PersistSmem {
 // DIR: directed graph (f4, reading R-9; also a separate instantiation).
 template <bool LA, bool DIR>
 __global__ __launch_bounds__(kPersistThreads, kPersistBlocks) void k_persist(
-    KArgs a, int* __restrict__ level, int* __restrict__ parent, const unsigned int* __restrict__ nonisolated,
-    long long nonisolated_count) {
+    KArgs a, const unsigned int* __restrict__ nonisolated, long long nonisolated_count) {
     extern __shared__ __align__(16) unsigned char dsm[];
     PersistSmem<LA>& sm = *reinterpret_cast<PersistSmem<LA>*>(dsm);
     __shared__ SelState s;
     unsigned epoch = 0;
     unsigned* bar = &a.st->bar_count;
+    int* __restrict__ level = a.st->out_level;
+    int* __restrict__ parent = a.st->out_parent;
+    if (threadIdx.x == 0) atomicMin(&a.st->t_enter, globaltimer());
     count_launch(a.st);
     // the source's entries are written by the fill itself and the seed state by one
     // thread alongside it: one barrier for both
@@ -1243,21 +1242,18 @@ Grids grids_for(const xbfs_graph* g) {
     return r;
 }
 
-// Optional per-launch event timing (xbfs_run_stats.kernel_capacity > 0).
+// Optional per-launch event timing (xbfs_run_stats.kernel_capacity > 0), from the
+// event pool the handle created at build time (at most kProfLaunches launches).
 struct Prof {
     xbfs_graph* g = nullptr;
     xbfs_run_stats* st = nullptr;
     int n = 0;
-    bool on() const { return st && st->kernel_capacity > 0 && n < st->kernel_capacity; }
+    bool on() const {
+        return st && st->kernel_capacity > 0 && n < st->kernel_capacity && 2 * (n + 1) <= (int)g->prof_events.size();
+    }
     xbfs_status before() {
         if (!on()) return XBFS_OK;
-        auto& ev = g->prof_events;
-        while ((int)ev.size() < 2 * (n + 1)) {
-            cudaEvent_t e;
-            XBFS_CUDA(g, cudaEventCreate(&e));
-            ev.push_back(e);
-        }
-        XBFS_CUDA(g, cudaEventRecord(ev[2 * n], g->stream));
+        XBFS_CUDA(g, cudaEventRecord(g->prof_events[2 * n], g->stream));
         return XBFS_OK;
     }
     xbfs_status after(int id, int level) {
@@ -1295,34 +1291,31 @@ struct Prof {
     } while (0)
 
 // Enqueue one level given the host-known strategy / queue state.
-xbfs_status launch_level(xbfs_graph* g, const KArgs& a, int* level, int* parent, int k, int strat,
-                         int queue_valid, long long fedges, unsigned maxdeg, int prev_small, long long small_edges,
-                         Prof& P) {
+xbfs_status launch_level(xbfs_graph* g, const KArgs& a, int k, int strat, int queue_valid, long long fedges,
+                         unsigned maxdeg, int prev_small, long long small_edges, Prof& P) {
     const Grids G = grids_for(g);
     cudaStream_t s = g->stream;
     // The small-frontier kernel advances the level state itself (no k_select).
     if (prev_small && small_gate(small_edges, strat, queue_valid, fedges, maxdeg)) {
-        XBFS_LAUNCH(P, XBFS_K_SMALL, k, (k_small_sf<<<kSmallCluster, kSmallThreads, 0, s>>>(a, level, parent)));
+        XBFS_LAUNCH(P, XBFS_K_SMALL, k, (k_small_sf<<<kSmallCluster, kSmallThreads, 0, s>>>(a)));
         return XBFS_OK;
     }
     if (strat != XBFS_BU && !queue_valid)
         XBFS_LAUNCH(P, XBFS_K_GENERATE_PRE, k, (k_generate<<<G.gen, kGenThreads, 0, s>>>(a, 0)));
     if (strat == XBFS_SF) {
-        XBFS_LAUNCH(P, XBFS_K_TD_SF, k,
-                    (k_td_expand<XBFS_SF><<<G.expand, kExpandThreads, 0, s>>>(a, level, parent)));
+        XBFS_LAUNCH(P, XBFS_K_TD_SF, k, (k_td_expand<XBFS_SF><<<G.expand, kExpandThreads, 0, s>>>(a)));
     } else if (strat == XBFS_SS) {
-        XBFS_LAUNCH(P, XBFS_K_TD_SS, k,
-                    (k_td_expand<XBFS_SS><<<G.expand, kExpandThreads, 0, s>>>(a, level, parent)));
+        XBFS_LAUNCH(P, XBFS_K_TD_SS, k, (k_td_expand<XBFS_SS><<<G.expand, kExpandThreads, 0, s>>>(a)));
         XBFS_LAUNCH(P, XBFS_K_SS_COUNT, k, (k_ss_count<<<G.gen, kGenThreads, 0, s>>>(a)));
     } else {
-        XBFS_LAUNCH(P, XBFS_K_BU, k, (k_bu_traverse<<<G.bu, kBuThreads, 0, s>>>(a, level, parent)));
+        XBFS_LAUNCH(P, XBFS_K_BU, k, (k_bu_traverse<<<G.bu, kBuThreads, 0, s>>>(a)));
     }
     XBFS_LAUNCH(P, XBFS_K_SELECT, k, (k_select<false><<<1, 1, 0, s>>>(a, 0)));
     return XBFS_OK;
 }
 
-xbfs_status run_host_loop(xbfs_graph* g, const KArgs& a, int* level, int* parent, long long small_edges,
-                          const int8_t* plan, int plan_len, Prof& P) {
+xbfs_status run_host_loop(xbfs_graph* g, const KArgs& a, long long small_edges, const int8_t* plan, int plan_len,
+                          Prof& P) {
     // k_seed wrote hctl; wait for it, then one sync per level (P:L151's
     // host/device crossing, kept as the debug / measurement driver).
     XBFS_CUDA(g, cudaStreamSynchronize(g->stream));
@@ -1339,18 +1332,19 @@ xbfs_status run_host_loop(xbfs_graph* g, const KArgs& a, int* level, int* parent
                                              g->stream));
             }
         }
-        XBFS_TRY(launch_level(g, a, level, parent, k, strat, h->queue_valid, h->fedges, h->fmaxdeg, prev_small,
-                              small_edges, P));
+        XBFS_TRY(launch_level(g, a, k, strat, h->queue_valid, h->fedges, h->fmaxdeg, prev_small, small_edges, P));
         XBFS_CUDA(g, cudaStreamSynchronize(g->stream));
     }
     return XBFS_OK;
 }
 
 // ------------------------------------------------- CUDA-graph device loop
-// One graph per (handle, level, parent): init -> seed -> WHILE(!done) {
-//   plan -> SWITCH{SF | gen+SF | SS+gen | gen+SS+gen | BU} -> select }.
-// The strategy decision never leaves the device: one launch per BFS instead of
-// one host/device crossing per level (the paper's P:L151 cost).
+// One graph per handle: init -> seed -> WHILE(!done) { plan -> SWITCH{SF | gen+SF |
+// SS+count | gen+SS+count | BU | small} -> select }.  The kernels take
+// the run's parameters and output pointers from the device state, so the graph is
+// instantiated once (xbfs_build_csr / xbfs_reorder), never inside xbfs_run.  The
+// strategy decision never leaves the device: one launch per BFS instead of one
+// host/device crossing per level (the paper's P:L151 cost).
 xbfs_status add_kernel(xbfs_graph* g, cudaGraph_t gr, cudaGraphNode_t* out, const cudaGraphNode_t* dep,
                        void* fn, int grid, int block, void** args) {
     cudaKernelNodeParams p = {};
@@ -1364,17 +1358,11 @@ xbfs_status add_kernel(xbfs_graph* g, cudaGraph_t gr, cudaGraphNode_t* out, cons
     return XBFS_OK;
 }
 
-xbfs_status build_loop_graph(xbfs_graph* g, int* level, int* parent) {
-    xbfs_graph::LoopGraph* slot = &g->loops[0];
-    for (auto& l : g->loops) {
-        if (l.exec && l.level == level && l.parent == parent) {
-            l.used = ++g->loop_tick;
-            g->cur_exec = l.exec;
-            return XBFS_OK;
-        }
-        if (l.used < slot->used) slot = &l;
+xbfs_status build_loop_graph(xbfs_graph* g) {
+    if (g->loop_exec) {
+        cudaGraphExecDestroy(g->loop_exec);
+        g->loop_exec = nullptr;
     }
-    if (slot->exec) { cudaGraphExecDestroy(slot->exec); *slot = xbfs_graph::LoopGraph(); }
     const Grids G = grids_for(g);
     KArgs a = g->kargs();
     const unsigned int* noniso = g->nonisolated;
@@ -1384,11 +1372,11 @@ xbfs_status build_loop_graph(xbfs_graph* g, int* level, int* parent) {
     struct Del { cudaGraph_t& t; ~Del() { if (t) cudaGraphDestroy(t); } } del{top};
     cudaGraphNode_t n_init, n_seed, n_while, n_plan, n_sw, n_sel, x, y;
     {
-        void* args[] = {&a, &level, &parent, &noniso};
+        void* args[] = {&a, &noniso};
         XBFS_TRY(add_kernel(g, top, &n_init, nullptr, (void*)k_init_fill, G.init, 256, args));
     }
     {
-        void* args[] = {&a, &level, &parent, &nic, &noniso};
+        void* args[] = {&a, &nic, &noniso};
         XBFS_TRY(add_kernel(g, top, &n_seed, &n_init, (void*)k_seed, 1, 1, args));
     }
     cudaGraphConditionalHandle h_while, h_switch;
@@ -1413,43 +1401,37 @@ xbfs_status build_loop_graph(xbfs_graph* g, int* level, int* parent) {
     XBFS_CUDA(g, cudaGraphAddNode(&n_sw, body, &n_plan, 1, &sp));
     cudaGraph_t* br = sp.conditional.phGraph_out;
     int role0 = 0;
-    void* a_exp[] = {&a, &level, &parent};
-    void* a_small[] = {&a, &level, &parent};
+    void* a_exp[] = {&a};
     void* a_gen0[] = {&a, &role0};
     void* f_sf = (void*)k_td_expand<XBFS_SF>;
     void* f_ss = (void*)k_td_expand<XBFS_SS>;
     void* f_gen = (void*)k_generate;
     void* f_cnt = (void*)k_ss_count;
-    void* a_cnt[] = {&a};
     // 0: SF (queue valid)
     XBFS_TRY(add_kernel(g, br[0], &x, nullptr, f_sf, G.expand, kExpandThreads, a_exp));
     // 1: generate + SF
     XBFS_TRY(add_kernel(g, br[1], &x, nullptr, f_gen, G.gen, kGenThreads, a_gen0));
     XBFS_TRY(add_kernel(g, br[1], &y, &x, f_sf, G.expand, kExpandThreads, a_exp));
-    // 2: SS + generate (No-Frontier-Generation: the queue exists)
+    // 2: SS + count (No-Frontier-Generation: the queue exists)
     XBFS_TRY(add_kernel(g, br[2], &x, nullptr, f_ss, G.expand, kExpandThreads, a_exp));
-    XBFS_TRY(add_kernel(g, br[2], &y, &x, f_cnt, G.gen, kGenThreads, a_cnt));
-    // 3: generate + SS + generate
+    XBFS_TRY(add_kernel(g, br[2], &y, &x, f_cnt, G.gen, kGenThreads, a_exp));
+    // 3: generate + SS + count
     XBFS_TRY(add_kernel(g, br[3], &x, nullptr, f_gen, G.gen, kGenThreads, a_gen0));
     XBFS_TRY(add_kernel(g, br[3], &y, &x, f_ss, G.expand, kExpandThreads, a_exp));
-    XBFS_TRY(add_kernel(g, br[3], &x, &y, f_cnt, G.gen, kGenThreads, a_cnt));
+    XBFS_TRY(add_kernel(g, br[3], &x, &y, f_cnt, G.gen, kGenThreads, a_exp));
     // 4: BU
     XBFS_TRY(add_kernel(g, br[4], &x, nullptr, (void*)k_bu_traverse, G.bu, kBuThreads, a_exp));
     // 5: small-frontier cluster mode (cluster dims are compiled into the kernel)
-    XBFS_TRY(add_kernel(g, br[5], &x, nullptr, (void*)k_small_sf, kSmallCluster, kSmallThreads, a_small));
+    XBFS_TRY(add_kernel(g, br[5], &x, nullptr, (void*)k_small_sf, kSmallCluster, kSmallThreads, a_exp));
     {
         void* args[] = {&a, &h_while};
         XBFS_TRY(add_kernel(g, body, &n_sel, &n_sw, (void*)k_select<true>, 1, 1, args));
     }
-    XBFS_CUDA(g, cudaGraphInstantiate(&slot->exec, top, 0));
-    slot->level = level;
-    slot->parent = parent;
-    slot->used = ++g->loop_tick;
-    g->cur_exec = slot->exec;
+    XBFS_CUDA(g, cudaGraphInstantiate(&g->loop_exec, top, 0));
     return XBFS_OK;
 }
 
-xbfs_status launch_persist(xbfs_graph* g, const KArgs& a, int* level, int* parent, bool lookahead) {
+xbfs_status launch_persist(xbfs_graph* g, const KArgs& a, bool lookahead) {
     static int occ[3][64];
     static bool init[3][64] = {{false}};
     const int dev = g->device & 63, v = lookahead ? 1 : (g->directed ? 2 : 0);
@@ -1469,13 +1451,38 @@ xbfs_status launch_persist(xbfs_graph* g, const KArgs& a, int* level, int* paren
     long long nic = g->nonisolated_count;
     KArgs ka = a;
     ka.track_max = 0;   // no small-frontier mode inside the persistent kernel
-    void* args[] = {&ka, &level, &parent, &noniso, &nic};
-    XBFS_CUDA(g, cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(kPersistThreads), args, smem,
-                                             g->stream));
+    void* args[] = {&ka, &noniso, &nic};
+    XBFS_CUDA(g, cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(kPersistThreads), args, smem, g->stream));
     return XBFS_OK;
 }
 
 }  // namespace
+
+// Everything a run needs beyond the CSR, created at build time so that xbfs_run
+// never allocates: the CUDA-graph device loop (re-instantiated after
+// every re-arrangement, which may move col), the host-output scratch slots and
+// copy stream, and the per-launch profiling event pool.
+xbfs_status prepare_drivers(xbfs_graph* g) {
+    XBFS_TRY(build_loop_graph(g));
+    if (!g->scratch_level) {
+        XBFS_CUDA(g, cudaMalloc(&g->scratch_level, 2 * g->n * sizeof(int)));
+        XBFS_CUDA(g, cudaMalloc(&g->scratch_parent, 2 * g->n * sizeof(int)));
+    }
+    if (!g->copy_stream) {
+        XBFS_CUDA(g, cudaStreamCreateWithFlags(&g->copy_stream, cudaStreamNonBlocking));
+        for (int s = 0; s < 2; ++s) {
+            XBFS_CUDA(g, cudaEventCreateWithFlags(&g->ev_done[s], cudaEventDisableTiming));
+            XBFS_CUDA(g, cudaEventCreateWithFlags(&g->ev_copied[s], cudaEventDisableTiming));
+        }
+    }
+    while ((int)g->prof_events.size() < 2 * kProfLaunches) {
+        cudaEvent_t e;
+        XBFS_CUDA(g, cudaEventCreate(&e));
+        g->prof_events.push_back(e);
+    }
+    return XBFS_OK;
+}
+
 }  // namespace xbfs
 
 using namespace xbfs;
@@ -1483,6 +1490,7 @@ using namespace xbfs;
 static xbfs_status run_impl(xbfs_graph* g, int64_t source, int32_t* level, int32_t* parent,
                             const xbfs_run_opts* opts, xbfs_run_stats* stats) {
     if (!g) return set_error(XBFS_ERR_INVALID_ARG, "xbfs_run: NULL handle");
+    if (g->dist) return set_error(XBFS_ERR_STATE, "xbfs_run: a distributed handle runs with xbfs_run_dist");
     if (!level || !parent) return set_error(XBFS_ERR_INVALID_ARG, "xbfs_run: NULL level/parent");
     if (source < 0 || source >= g->n)
         return set_error(XBFS_ERR_INVALID_ARG, "xbfs_run: source %lld outside [0, %lld)", (long long)source, g->n);
@@ -1492,10 +1500,10 @@ static xbfs_status run_impl(xbfs_graph* g, int64_t source, int32_t* level, int32
     if (opts) o = *opts;
     if (o.force_strategy < -1 || o.force_strategy > 2)
         return set_error(XBFS_ERR_INVALID_ARG, "force_strategy must be -1..2");
+    if (o.driver < 0 || o.driver > 3) return set_error(XBFS_ERR_INVALID_ARG, "driver must be 0..3");
     XBFS_CUDA(g, cudaSetDevice(g->device));
 
     KArgs a = g->kargs();
-    if (o.driver < 0 || o.driver > 3) return set_error(XBFS_ERR_INVALID_ARG, "driver must be 0..3");
     const bool host_only = (stats && stats->kernel_capacity > 0) || (o.plan && o.plan_len > 0);
     const bool use_persist = (o.driver == 0 || o.driver == 3) && !host_only;
     const bool use_graph = o.driver == 2 && !host_only;
@@ -1505,7 +1513,7 @@ static xbfs_status run_impl(xbfs_graph* g, int64_t source, int32_t* level, int32
                          "profiling, no look-ahead)");
     if (o.lookahead && !use_persist)
         return set_error(XBFS_ERR_INVALID_ARG, "lookahead needs the persistent driver (driver 0/3, no plan/profiling)");
-    // selection parameters live in the device state
+    // selection parameters and output pointers live in the device state
     {
         DevState hs;
         memset(&hs, 0, sizeof(hs));
@@ -1518,6 +1526,9 @@ static xbfs_status run_impl(xbfs_graph* g, int64_t source, int32_t* level, int32
         hs.small_edges = std::min<long long>(std::max(o.small_edges, 0), kSmallEdgesMax);
         hs.mirror_host = (use_graph || use_persist) ? 0 : 1;
         hs.lookahead = o.lookahead ? 1 : 0;
+        hs.out_level = level;
+        hs.out_parent = parent;
+        hs.t_enter = ~0ull;
         XBFS_CUDA(g, cudaMemcpyAsync(g->st, &hs, sizeof(hs), cudaMemcpyHostToDevice, g->stream));
     }
     const Grids G = grids_for(g);
@@ -1526,22 +1537,20 @@ static xbfs_status run_impl(xbfs_graph* g, int64_t source, int32_t* level, int32
     P.st = stats;
     if (use_persist) {
         XBFS_CUDA(g, cudaEventRecord(g->ev0, g->stream));
-        XBFS_TRY(launch_persist(g, a, level, parent, o.lookahead != 0));
+        XBFS_TRY(launch_persist(g, a, o.lookahead != 0));
         XBFS_CUDA(g, cudaEventRecord(g->ev1, g->stream));
     } else if (use_graph) {
-        XBFS_TRY(build_loop_graph(g, level, parent));
         XBFS_CUDA(g, cudaEventRecord(g->ev0, g->stream));
-        XBFS_CUDA(g, cudaGraphLaunch(g->cur_exec, g->stream));
+        XBFS_CUDA(g, cudaGraphLaunch(g->loop_exec, g->stream));
         XBFS_CUDA(g, cudaEventRecord(g->ev1, g->stream));
     } else {
-    XBFS_CUDA(g, cudaEventRecord(g->ev0, g->stream));
-    XBFS_LAUNCH(P, XBFS_K_INIT, -1,
-                (k_init_fill<<<G.init, 256, 0, g->stream>>>(a, level, parent, g->nonisolated)));
-    XBFS_LAUNCH(P, XBFS_K_SEED, -1,
-                (k_seed<<<1, 1, 0, g->stream>>>(a, level, parent, g->nonisolated_count, g->nonisolated)));
-    XBFS_TRY(run_host_loop(g, a, level, parent, std::min<long long>(std::max(o.small_edges, 0), kSmallEdgesMax),
-                           o.plan, o.plan ? std::max(o.plan_len, 0) : 0, P));
-    XBFS_CUDA(g, cudaEventRecord(g->ev1, g->stream));
+        XBFS_CUDA(g, cudaEventRecord(g->ev0, g->stream));
+        XBFS_LAUNCH(P, XBFS_K_INIT, -1, (k_init_fill<<<G.init, 256, 0, g->stream>>>(a, g->nonisolated)));
+        XBFS_LAUNCH(P, XBFS_K_SEED, -1,
+                    (k_seed<<<1, 1, 0, g->stream>>>(a, g->nonisolated_count, g->nonisolated)));
+        XBFS_TRY(run_host_loop(g, a, std::min<long long>(std::max(o.small_edges, 0), kSmallEdgesMax), o.plan,
+                               o.plan ? std::max(o.plan_len, 0) : 0, P));
+        XBFS_CUDA(g, cudaEventRecord(g->ev1, g->stream));
     }
 
     if (stats) {
@@ -1561,26 +1570,39 @@ static xbfs_status run_impl(xbfs_graph* g, int64_t source, int32_t* level, int32
         stats->arcs_traversed = hs.arcs_traversed;
         stats->input_edges_traversed = (int64_t)m;
         stats->kernel_launches = hs.launches;
+        // persistent driver: first CTA entry .. end of init + seed (%globaltimer)
+        stats->init_ms = (use_persist && hs.t_enter != ~0ull && hs.t_start >= hs.t_enter)
+                             ? (float)((hs.t_start - hs.t_enter) * 1e-6) : 0.f;
         XBFS_TRY(P.finish());
         const int nl = std::min(hs.nlevels, std::min(stats->level_capacity, kLogCap));
         if (nl > 0 && (stats->strategy || stats->frontier_vertices || stats->frontier_edges ||
                        stats->unvisited || stats->bu_probes || stats->level_ms || stats->lookahead_found)) {
-            LevelRec* rec = new LevelRec[nl];
-            XBFS_CUDA(g, cudaMemcpy(rec, g->log, nl * sizeof(LevelRec), cudaMemcpyDeviceToHost));
-            for (int i = 0; i < nl; ++i) {
-                if (stats->strategy) stats->strategy[i] = (int8_t)rec[i].strategy;
-                if (stats->frontier_vertices) stats->frontier_vertices[i] = rec[i].fsize;
-                if (stats->frontier_edges) stats->frontier_edges[i] = rec[i].fedges;
-                if (stats->unvisited) stats->unvisited[i] = rec[i].unvisited;
-                if (stats->bu_probes) stats->bu_probes[i] = rec[i].probes;
-                if (stats->lookahead_found) stats->lookahead_found[i] = rec[i].la_found;
-                if (stats->level_ms) {
-                    const unsigned long long t0 = i ? rec[i - 1].t_ns : hs.t_start;
-                    stats->level_ms[i] = (use_persist && rec[i].t_ns >= t0 && t0) ? (float)((rec[i].t_ns - t0) * 1e-6)
-                                                                                   : 0.f;
+            // the log is copied in slices through a fixed host buffer (no allocation per run)
+            LevelRec rec[256];
+            for (int i0 = 0; i0 < nl; i0 += 256) {
+                const int cnt = std::min(256, nl - i0);
+                XBFS_CUDA(g, cudaMemcpy(rec, g->log + i0, cnt * sizeof(LevelRec), cudaMemcpyDeviceToHost));
+                for (int j = 0; j < cnt; ++j) {
+                    const int i = i0 + j;
+                    const LevelRec& r = rec[j];
+                    if (stats->strategy) stats->strategy[i] = (int8_t)r.strategy;
+                    if (stats->frontier_vertices) stats->frontier_vertices[i] = r.fsize;
+                    if (stats->frontier_edges) stats->frontier_edges[i] = r.fedges;
+                    if (stats->unvisited) stats->unvisited[i] = r.unvisited;
+                    if (stats->bu_probes) stats->bu_probes[i] = r.probes;
+                    if (stats->lookahead_found) stats->lookahead_found[i] = r.la_found;
+                    if (stats->level_ms) {
+                        unsigned long long t0 = hs.t_start;
+                        if (i > 0) {
+                            LevelRec prev;
+                            if (j > 0) prev = rec[j - 1];
+                            else XBFS_CUDA(g, cudaMemcpy(&prev, g->log + i - 1, sizeof(LevelRec), cudaMemcpyDeviceToHost));
+                            t0 = prev.t_ns;
+                        }
+                        stats->level_ms[i] = (use_persist && r.t_ns >= t0 && t0) ? (float)((r.t_ns - t0) * 1e-6) : 0.f;
+                    }
                 }
             }
-            delete[] rec;
         }
     }
     return XBFS_OK;
@@ -1591,25 +1613,18 @@ extern "C" xbfs_status xbfs_run(xbfs_graph* g, int64_t source, int32_t* level, i
     return run_impl(g, source, level, parent, opts, stats);
 }
 
-// Two device output slots + a copy stream for the host-output calls (lazily, 16N bytes).
-static xbfs_status ensure_host_scratch(xbfs_graph* g) {
-    if (!g->scratch_level) {
-        XBFS_CUDA(g, cudaMalloc(&g->scratch_level, 2 * g->n * sizeof(int)));
-        XBFS_CUDA(g, cudaMalloc(&g->scratch_parent, 2 * g->n * sizeof(int)));
-    }
-    if (!g->copy_stream) {
-        XBFS_CUDA(g, cudaStreamCreateWithFlags(&g->copy_stream, cudaStreamNonBlocking));
-        for (int s = 0; s < 2; ++s) {
-            XBFS_CUDA(g, cudaEventCreateWithFlags(&g->ev_done[s], cudaEventDisableTiming));
-            XBFS_CUDA(g, cudaEventCreateWithFlags(&g->ev_copied[s], cudaEventDisableTiming));
-        }
-    }
-    return XBFS_OK;
+// A failing host-output call must not return while copies it enqueued can still
+// write into the caller's host buffers: drain both streams first (best effort).
+static xbfs_status drain(xbfs_graph* g, xbfs_status s) {
+    if (g->copy_stream) cudaStreamSynchronize(g->copy_stream);
+    if (g->stream) cudaStreamSynchronize(g->stream);
+    return s;
 }
 
 extern "C" xbfs_status xbfs_run_host_batch(xbfs_graph* g, const int64_t* sources, int32_t count, int32_t host_slots,
                                            int32_t* level_host, int32_t* parent_host, const xbfs_run_opts* opts) {
     if (!g) return set_error(XBFS_ERR_INVALID_ARG, "xbfs_run_host_batch: NULL handle");
+    if (g->dist) return set_error(XBFS_ERR_STATE, "xbfs_run_host_batch: distributed handle");
     if (count < 0 || host_slots < 1) return set_error(XBFS_ERR_INVALID_ARG, "xbfs_run_host_batch: count < 0 or host_slots < 1");
     if (count == 0) return XBFS_OK;
     if (!sources || !level_host || !parent_host)
@@ -1620,21 +1635,24 @@ extern "C" xbfs_status xbfs_run_host_batch(xbfs_graph* g, const int64_t* sources
                              (long long)sources[i], g->n);
     if (g->poisoned) return set_error(XBFS_ERR_STATE, "handle poisoned by an earlier failure");
     XBFS_CUDA(g, cudaSetDevice(g->device));
-    XBFS_TRY(ensure_host_scratch(g));
     const size_t bytes = (size_t)g->n * sizeof(int);
     for (int32_t i = 0; i < count; ++i) {
         const int s = i & 1;
         int* lv = g->scratch_level + (size_t)s * g->n;
         int* pa = g->scratch_parent + (size_t)s * g->n;
+        cudaError_t e = cudaSuccess;
         // slot s is free once the D2H copies of BFS i-2 have drained
-        if (i >= 2) XBFS_CUDA(g, cudaStreamWaitEvent(g->stream, g->ev_copied[s], 0));
-        XBFS_TRY(run_impl(g, sources[i], lv, pa, opts, nullptr));
-        XBFS_CUDA(g, cudaEventRecord(g->ev_done[s], g->stream));
-        XBFS_CUDA(g, cudaStreamWaitEvent(g->copy_stream, g->ev_done[s], 0));
+        if (i >= 2) e = cudaStreamWaitEvent(g->stream, g->ev_copied[s], 0);
+        if (e != cudaSuccess) return drain(g, cuda_fail(g, e, "cudaStreamWaitEvent"));
+        xbfs_status st = run_impl(g, sources[i], lv, pa, opts, nullptr);
+        if (st != XBFS_OK) return drain(g, st);
         const size_t off = (size_t)(i % host_slots) * g->n;
-        XBFS_CUDA(g, cudaMemcpyAsync(level_host + off, lv, bytes, cudaMemcpyDeviceToHost, g->copy_stream));
-        XBFS_CUDA(g, cudaMemcpyAsync(parent_host + off, pa, bytes, cudaMemcpyDeviceToHost, g->copy_stream));
-        XBFS_CUDA(g, cudaEventRecord(g->ev_copied[s], g->copy_stream));
+        if ((e = cudaEventRecord(g->ev_done[s], g->stream)) != cudaSuccess ||
+            (e = cudaStreamWaitEvent(g->copy_stream, g->ev_done[s], 0)) != cudaSuccess ||
+            (e = cudaMemcpyAsync(level_host + off, lv, bytes, cudaMemcpyDeviceToHost, g->copy_stream)) != cudaSuccess ||
+            (e = cudaMemcpyAsync(parent_host + off, pa, bytes, cudaMemcpyDeviceToHost, g->copy_stream)) != cudaSuccess ||
+            (e = cudaEventRecord(g->ev_copied[s], g->copy_stream)) != cudaSuccess)
+            return drain(g, cuda_fail(g, e, "xbfs_run_host_batch copy-back"));
     }
     XBFS_CUDA(g, cudaStreamSynchronize(g->copy_stream));
     XBFS_CUDA(g, cudaStreamSynchronize(g->stream));
@@ -1644,12 +1662,12 @@ extern "C" xbfs_status xbfs_run_host_batch(xbfs_graph* g, const int64_t* sources
 extern "C" xbfs_status xbfs_run_host(xbfs_graph* g, int64_t source, int32_t* level_host, int32_t* parent_host,
                                      const xbfs_run_opts* opts, xbfs_run_stats* stats) {
     if (!g) return set_error(XBFS_ERR_INVALID_ARG, "xbfs_run_host: NULL handle");
+    if (g->dist) return set_error(XBFS_ERR_STATE, "xbfs_run_host: distributed handle");
     if (!level_host || !parent_host) return set_error(XBFS_ERR_INVALID_ARG, "xbfs_run_host: NULL level/parent");
     if (g->poisoned) return set_error(XBFS_ERR_STATE, "handle poisoned by an earlier failure");
     XBFS_CUDA(g, cudaSetDevice(g->device));
-    XBFS_TRY(ensure_host_scratch(g));
     xbfs_status s = run_impl(g, source, g->scratch_level, g->scratch_parent, opts, stats);
-    if (s != XBFS_OK) return s;
+    if (s != XBFS_OK) return drain(g, s);
     XBFS_CUDA(g, cudaMemcpyAsync(level_host, g->scratch_level, g->n * sizeof(int), cudaMemcpyDeviceToHost, g->stream));
     XBFS_CUDA(g, cudaMemcpyAsync(parent_host, g->scratch_parent, g->n * sizeof(int), cudaMemcpyDeviceToHost, g->stream));
     XBFS_CUDA(g, cudaStreamSynchronize(g->stream));

@@ -449,6 +449,8 @@ extern "C" xbfs_status xbfs_build_csr(const void* src, const void* dst, int64_t 
     }
     if ((unsigned long long)arcs >= (1ull << g->dbits))
         return set_error(XBFS_ERR_INVALID_ARG, "graph too large for the packed queue counter");
+    XBFS_TRY_B(prepare_drivers(g));
+    XBFS_CUDA(g, cudaStreamSynchronize(g->stream));
     guard.keep = true;
     *out = g;
     return XBFS_OK;
@@ -470,8 +472,8 @@ extern "C" xbfs_status xbfs_reorder(xbfs_graph* g, int32_t mode) {
     k_head<<<grid_for(n), kB, 0, g->stream>>>(g->row_ptr, g->col, n, g->head, g->head32, g->idbits);
     XBFS_CUDA(g, cudaGetLastError());
     XBFS_CUDA(g, cudaStreamSynchronize(g->stream));
-    // the BFS graph (if any) captured the old col pointer
-    g->drop_loops();
+    // the device-loop graph captured the old col pointer: re-instantiate it here (never in xbfs_run)
+    XBFS_TRY_B(prepare_drivers(g));
     g->reorder_mode = mode;
     return XBFS_OK;
 }

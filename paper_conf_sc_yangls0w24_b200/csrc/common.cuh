@@ -41,6 +41,7 @@ constexpr int kSmallBig = 8192;      // per-CTA list of higher-degree vertices (
 constexpr long long kSmallEdgesMax = 9LL * kSmallBig;  // guarantees the big list never overflows
 constexpr int kSmallMaxDeg = 512;    // frontier max degree allowed in the small mode (warp steps <= 16)
 constexpr int kLogCap = 1 << 16;     // per-level log entries kept on the device
+constexpr int kProfLaunches = 4096;  // per-launch timing: launches recorded at most
 #ifndef XBFS_PERSIST_THREADS
 #define XBFS_PERSIST_THREADS 1024
 #endif
@@ -95,6 +96,9 @@ struct DevState {
     int mirror_host;             // host-loop driver: mirror the level state into HostCtl
     int lookahead;               // BU look-ahead (persistent driver)
     unsigned long long t_start;  // %globaltimer after init + seed (persistent driver)
+    unsigned long long t_enter;  // earliest CTA entry of the persistent kernel (atomicMin; host sets ~0)
+    int* out_level;              // the run's output arrays (set per run with the parameters; the
+    int* out_parent;             // per-level kernels read them here, so one CUDA graph serves any outputs)
     // persistent driver: grid-barrier arrival counter, alone on its 128-byte line
     // (zeroed with the rest of the state before every run)
     alignas(128) unsigned bar_count;
@@ -176,27 +180,15 @@ struct xbfs_graph {
     cudaEvent_t ev_done[2] = {nullptr, nullptr}, ev_copied[2] = {nullptr, nullptr};
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
     int dbits = 40;
-    // CUDA-graph device loop (built lazily)
-    struct LoopGraph {
-        cudaGraphExec_t exec = nullptr;
-        int* level = nullptr;            // output pointers the graph was built for
-        int* parent = nullptr;
-        unsigned long long used = 0;
-    };
-    LoopGraph loops[4];                  // small LRU cache of instantiated device loops
-    unsigned long long loop_tick = 0;
-    cudaGraphExec_t cur_exec = nullptr;
-    void drop_loops() {
-        for (auto& l : loops) {
-            if (l.exec) cudaGraphExecDestroy(l.exec);
-            l = LoopGraph();
-        }
-    }
-    std::vector<cudaEvent_t> prof_events;  // per-launch timing pool
+    cudaGraphExec_t loop_exec = nullptr;   // CUDA-graph device loop: one per handle, built with it
+    std::vector<cudaEvent_t> prof_events;  // per-launch timing pool (2 * kProfLaunches, built with it)
+    struct xbfs_dist_part* dist = nullptr; // multi-GPU partition (xbfs_build_csr_dist); NULL = single GPU
     xbfs::KArgs kargs() const;
 };
 
 namespace xbfs {
+// driver state created at build / re-arrangement time (bfs.cu)
+xbfs_status prepare_drivers(xbfs_graph* g);
 // error plumbing (api.cu)
 xbfs_status set_error(xbfs_status s, const char* fmt, ...);
 xbfs_status cuda_fail(xbfs_graph* g, cudaError_t e, const char* what);

@@ -57,7 +57,8 @@ class RunStats(ctypes.Structure):
                 ("kernel_capacity", ctypes.c_int32), ("num_kernels", ctypes.c_int32),
                 ("kernel_id", ctypes.POINTER(ctypes.c_int32)), ("kernel_level", ctypes.POINTER(ctypes.c_int32)),
                 ("kernel_ms", ctypes.POINTER(ctypes.c_float)), ("level_ms", ctypes.POINTER(ctypes.c_float)),
-                ("lookahead_found", ctypes.POINTER(ctypes.c_int64))]
+                ("lookahead_found", ctypes.POINTER(ctypes.c_int64)),
+                ("init_ms", ctypes.c_float)]
 
 
 #: kernel ids of RunStats.kernel_id (XBFS_K_* in include/xbfs.h)
@@ -137,7 +138,18 @@ def xbfs_run(g: int, source: int, level, parent, opts: RunOpts | None = None, st
                         ctypes.byref(stats) if stats else None))
 
 
+def _check_host_out(level, parent, need: int):
+    """The C side DMAs straight into these buffers and cannot bound-check them:
+    int32, C-contiguous host arrays of at least `need` elements each."""
+    for name, a in (("level", level), ("parent", parent)):
+        if not isinstance(a, np.ndarray) or a.dtype != np.int32 or not a.flags["C_CONTIGUOUS"]:
+            raise TypeError(f"{name}: need a C-contiguous int32 numpy array (host memory)")
+        if a.size < need:
+            raise ValueError(f"{name}: {a.size} elements < the {need} the call writes")
+
+
 def xbfs_run_host(g: int, source: int, level, parent, opts: RunOpts | None = None, stats: RunStats | None = None):
+    _check_host_out(level, parent, xbfs_graph_info(g)[0])
     _check(lib.xbfs_run_host(g, source, _ptr(level), _ptr(parent), ctypes.byref(opts) if opts else None,
                              ctypes.byref(stats) if stats else None))
 
@@ -149,6 +161,9 @@ def xbfs_run_host_batch(g: int, sources, level, parent, host_slots: int | None =
     src = np.ascontiguousarray(np.asarray(sources, dtype=np.int64))
     k = int(src.size)
     slots = k if host_slots is None else int(host_slots)
+    if k:
+        n = xbfs_graph_info(g)[0]
+        _check_host_out(level, parent, max(slots, 1) * n)
     _check(lib.xbfs_run_host_batch(g, src.ctypes.data if k else None, k, max(slots, 1) if k == 0 else slots,
                                    _ptr(level), _ptr(parent), ctypes.byref(opts) if opts else None))
 
@@ -192,6 +207,7 @@ class Stats:
     kernels: list = field(default_factory=list)   # (name, level, ms) when profiled
     level_ms: list = field(default_factory=list)  # device ms per level (persistent driver)
     lookahead_found: list = field(default_factory=list)  # level-(k+2) vertices set by BU step k
+    init_ms: float = 0.0        # persistent driver: kernel entry .. end of init + seed (device time)
 
 
 class _StatsBuf:
@@ -232,7 +248,7 @@ class _StatsBuf:
                      self.un[:nl].tolist(), self.pr[:nl].tolist(),
                      [(KERNEL_NAMES[int(self.kid[i])], int(self.klv[i]), float(self.kms[i]))
                       for i in range(min(c.num_kernels, self.kcap))] if self.kcap else [],
-                     self.lms[:nl].tolist(), self.laf[:nl].tolist())
+                     self.lms[:nl].tolist(), self.laf[:nl].tolist(), c.init_ms)
 
 
 def make_run_opts(alpha=None, grow=None, ratio_min=None, bu_stay=None, force_strategy=None, driver=None,

@@ -1,6 +1,8 @@
 """GPU parity for directed graphs (reading R-9): the CUDA path
 through the C ABI against the oracle's out-arc CSR, textbook BFS and arc-wise
-Graph500 validation.  Levels must match BIT-EXACTLY; parents must validate;
+Graph500 validation.  Levels must match BIT-EXACTLY; parents must validate and
+equal reading R-12's choice (the first in-neighbour of the re-arranged in-arc
+row one level up, oracle_first_parents) BIT-EXACTLY;
 the per-level counters (|F_k|, edgesF_k over OUT-degrees), vertices reached,
 arcs traversed and Graph500 m must equal the oracle's.  Every strategy is
 forced on every level besides the adaptive selector, so the in-arc bottom-up
@@ -29,12 +31,39 @@ def _dev(a):
     return torch.from_numpy(np.ascontiguousarray(a).view(np.int32)).cuda()
 
 
+_ROWS = {}
+
+
+def in_rows(og, src, dst, reordered=True):
+    """R-12 parent rows of a directed graph: the in-arc CSR, re-arranged by the
+    in-neighbour's out-degree (R-9) when the library's graph is (cached)."""
+    key = (id(og), reordered)
+    if key not in _ROWS or _ROWS[key][0] is not og:
+        t = oracle.transpose_directed(og.n, src, dst)
+        _ROWS[key] = (og, oracle.reorder(t, deg_from=og) if reordered else t)
+    return _ROWS[key][1]
+
+
+def check_parents_directed(og, src, dst, root, lv, pa, reordered=True, strategy=None):
+    """Parents: arc-wise V1-V5 everywhere; R-12 exact where a bottom-up step found the vertex."""
+    assert oracle.validate_directed(og, src, dst, int(root), lv, pa) == 0, f"validation (root {root})"
+    want, orphans = oracle.first_parents(in_rows(og, src, dst, reordered), lv, int(root))
+    assert orphans == 0
+    exact = lv <= 1
+    if strategy is not None:
+        st = np.asarray(list(strategy) + [-1], dtype=np.int64)
+        idx = np.clip(lv - 1, 0, len(st) - 1)
+        exact |= (lv >= 2) & (lv - 1 < len(strategy)) & (st[idx] == 2)
+    bad = np.flatnonzero(exact & (want != pa))
+    assert bad.size == 0, f"parents differ from R-12 at {bad[:5]} (root {root})"
+
+
 def _check(g, og, src, dst, root, **opts):
     level, parent, st = g.run(int(root), stats=True, **opts)
     lv, pa = level.cpu().numpy(), parent.cpu().numpy()
     ref, _, nl = oracle.bfs(og, int(root))
     assert np.array_equal(lv, ref), f"levels differ (root {root}, {opts})"
-    assert oracle.validate_directed(og, src, dst, int(root), lv, pa) == 0, f"validation (root {root}, {opts})"
+    check_parents_directed(og, src, dst, root, lv, pa, g.reordered, st.strategy)
     fs, fe = oracle.level_stats(og, ref)
     assert st.num_levels == nl
     cap = len(st.frontier_vertices)
@@ -220,5 +249,5 @@ def test_directed_int64_device_edges_and_host_batch(xb):
     for i, r in enumerate(roots):
         ref, _, _ = oracle.bfs(og, r)
         assert np.array_equal(lh[i * n:(i + 1) * n], ref)
-        assert oracle.validate_directed(og, src, dst, r, lh[i * n:(i + 1) * n], ph[i * n:(i + 1) * n]) == 0
+        check_parents_directed(og, src, dst, r, lh[i * n:(i + 1) * n], ph[i * n:(i + 1) * n])
     g.close()

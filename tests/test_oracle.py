@@ -599,3 +599,55 @@ def test_validate_tuples_random_graphs(seed):
             (oracle.validate(g, src, dst, int(s), lvd, pad) == 0)
         assert (oracle.validate_tuples(n, src, dst, int(s), lv, pa, directed=True) == 0) == \
             (oracle.validate_directed(gd, src, dst, int(s), lv, pa) == 0)
+
+
+# ------------------------------------------ R-12: deterministic first parents
+
+def test_first_parents_hand_computed():
+    """Reading R-12: parent[v] = the first vertex of v's RE-ARRANGED row one level up.
+    Diamond 0-1, 0-2, 1-3, 2-3 plus 2-4 from s = 0: levels 0,1,1,2,2; deg(2) = 3 >
+    deg(1) = 2, so row 3 is [2, 1] and parent[3] = 2 (id order would give 1).
+    Without 2-4 the degrees tie and the id-ascending tie-break gives 1."""
+    n, src, dst = _graph(5, [(0, 1), (0, 2), (1, 3), (2, 3), (2, 4)])
+    g = oracle.reorder(oracle.build_csr(n, src, dst))
+    level, _, _ = oracle.bfs(g, 0)
+    par, orphans = oracle.first_parents(g, level, 0)
+    assert par.tolist() == [0, 0, 0, 2, 2] and orphans == 0
+    n, src, dst = _graph(5, [(0, 1), (0, 2), (1, 3), (2, 3)])
+    g = oracle.reorder(oracle.build_csr(n, src, dst))
+    level, _, _ = oracle.bfs(g, 0)
+    par, _ = oracle.first_parents(g, level, 0)
+    assert par.tolist() == [0, 0, 0, 1, -1]
+    # path from 0: parent[v] = v - 1 (closed form)
+    n, src, dst = _graph(9, [(i, i + 1) for i in range(8)])
+    g = oracle.reorder(oracle.build_csr(n, src, dst))
+    level, _, _ = oracle.bfs(g, 0)
+    assert oracle.first_parents(g, level, 0)[0].tolist() == [0] + list(range(8))
+    # directed (R-9): in-arc row of 3 = {1, 2} ordered by OUT-degree (2 has 2, 1 has 1)
+    n, src, dst = _graph(5, [(0, 1), (0, 2), (1, 3), (2, 3), (2, 4)])
+    gd = oracle.build_csr_directed(n, src, dst)
+    tin = oracle.reorder(oracle.transpose_directed(n, src, dst), deg_from=gd)
+    assert tin.col[tin.row_ptr[3]:tin.row_ptr[4]].tolist() == [2, 1]
+    lv, _, _ = oracle.bfs(gd, 0)
+    assert oracle.first_parents(tin, lv, 0)[0].tolist() == [0, 0, 0, 2, 2]
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_first_parents_are_valid_bfs_parents(seed):
+    """On random graphs the R-12 parents pass Graph500 validation (V1-V5) and no
+    reached vertex is left without a parent; directed likewise over in-arc rows."""
+    rng = np.random.default_rng(1300 + seed)
+    n = int(rng.integers(2, 400))
+    e = rng.integers(0, n, (int(rng.integers(1, 5 * n)), 2))
+    n, src, dst = _graph(n, e)
+    g = oracle.build_csr(n, src, dst)
+    r = oracle.reorder(g)
+    gd = oracle.build_csr_directed(n, src, dst)
+    tin = oracle.reorder(oracle.transpose_directed(n, src, dst), deg_from=gd)
+    for s in rng.integers(0, n, 5):
+        lv, _, _ = oracle.bfs(g, int(s))
+        par, orphans = oracle.first_parents(r, lv, int(s))
+        assert orphans == 0 and oracle.validate(g, src, dst, int(s), lv, par) == 0
+        lvd, _, _ = oracle.bfs(gd, int(s))
+        pard, orphans = oracle.first_parents(tin, lvd, int(s))
+        assert orphans == 0 and oracle.validate_directed(gd, src, dst, int(s), lvd, pard) == 0

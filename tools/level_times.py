@@ -41,7 +41,8 @@ def main():
         flush.fill_(1)
         torch.cuda.synchronize()
         _, _, st = g.run(int(r), level, parent, stats=True, **opts)
-        print(f"root {int(r)}: {st.elapsed_ms * 1e3:.1f} us total, levels sum {sum(st.level_ms) * 1e3:.1f} us")
+        print(f"root {int(r)}: {st.elapsed_ms * 1e3:.1f} us total, levels sum {sum(st.level_ms) * 1e3:.1f} us, "
+              f"init {st.init_ms * 1e3:.1f} us")
         for k in range(st.num_levels):
             print(f"  L{k} {'FSB'[st.strategy[k]]} |F|={st.frontier_vertices[k]:>9,} ratio={st.frontier_edges[k] / g.arcs:9.3g} "
                   f"U={st.unvisited[k]:>10,} probes={st.bu_probes[k]:>11,} {st.level_ms[k] * 1e3:8.1f} us")
