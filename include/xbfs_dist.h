@@ -1,29 +1,33 @@
 /*
- * xbfs_dist.h — multi-GPU XBFS: 1D vertex partition, one process per GPU
- * (north_star: "for 2, 4 and 8 GPUs the graph is
- * 1D-partitioned by vertex ... with the direction switch made on globally
- * reduced counts").  The paper runs a single GCD and presents itself as
- * the basis for distributed BFS; the exchange below is this build's.
+ * xbfs_dist.h — multi-GPU XBFS: 1D vertex partition, one process per GPU on one
+ * node (SURVEY §8(a) row a11, §8(b) multi-GPU calls, §8(e); north_star: "for 2, 4
+ * and 8 GPUs the graph is 1D-partitioned by vertex ... with the direction switch
+ * made on globally reduced counts").  The paper runs a single GCD and
+ * presents itself as the basis for distributed BFS; the exchange below is
+ * this build's (reading R-10 in DESIGN.md).
  *
  * Partition: rank r owns vertices [r*B, min(N, (r+1)*B)), B = 32*ceil(N/(32p)),
- * with the full adjacency row (global neighbour ids) of every owned vertex.
+ * with the full adjacency row (global neighbour ids) of every owned vertex, rows
+ * re-arranged by neighbour degree descending, ties id ascending (C-12) —
+ * the true degrees, so every row is the single-GPU xbfs_reorder row.
  * Replicated per rank: three N-bit frontier bitmaps (F_k, F_{k+1}, stale).
- * Per level k (the strategy is identical on every rank, chosen from the
- * all-reduced counters by the paper's rule):
- *   BU  phase 0: owned unvisited vertices probe their neighbours in the local
- *       replica of F_k; the owned words of F_{k+1} are stored straight into every
- *       peer's replica (peer memory over NVLink/NVSwitch, CUDA IPC): the
- *       all-gather is fused into the producing kernel.
- *   TD  phase 0: owned frontier vertices expand their rows; an owned neighbour is
- *       claimed locally, a remote one is OR-ed into its owner's inbox bitmap in
- *       peer memory (fire-and-forget RED).  phase 1 (after a barrier): each owner
- *       turns inbox ∧ ¬visited into new frontier vertices, finds each one's parent
- *       with a bottom-up probe against F_k, and stores its owned F_{k+1} words
- *       into every peer's replica.
- * Host barriers and the 4-counter all-reduce between phases are the caller's
- * (torch.distributed), see paper_conf_sc_yangls0w24_b200/xbfs.py DistGraph.
+ * Per level k (the strategy is identical on every rank: the paper's rule, P:L87,
+ * on the all-reduced counters):
+ *   BU  owned unvisited vertices probe their rows against the local replica of
+ *       F_k; the owned words of F_{k+1} are stored straight into every peer's
+ *       replica (peer memory over NVLink/NVSwitch, CUDA IPC): the all-gather is
+ *       fused into the producing kernel.
+ *   TD  owned frontier vertices expand their rows; an owned neighbour is claimed
+ *       locally, a remote one is OR-ed into its owner's inbox bitmap in peer memory
+ *       (fire-and-forget RED); after a barrier each owner turns inbox ∧ ¬visited
+ *       into new frontier vertices, gives each the first vertex of its row in F_k
+ *       as parent, and stores its owned F_{k+1} words into every replica.
+ * The level loop, the barriers and the counter all-reduce run inside
+ * xbfs_run_dist (one C call per BFS); the host collectives use the communicator
+ * below (a shared-memory segment on the node, no NCCL: reading R-10).
  *
- * Conventions as in xbfs.h (status codes, thread-local error, poisoning).
+ * Conventions as in xbfs.h (status codes, thread-local error, handle poisoning;
+ * every call here is collective unless marked local).
  */
 #ifndef XBFS_DIST_H
 #define XBFS_DIST_H
@@ -36,66 +40,62 @@
 extern "C" {
 #endif
 
-#define XBFS_IPC_HANDLE_BYTES 64
+#define XBFS_UNIQUE_ID_BYTES 128
 #define XBFS_DIST_MAX_RANKS 16
-#define XBFS_DIST_NCOUNTS 8   /* length of every counts[] array below */
 
-typedef struct xbfs_dist xbfs_dist;
+typedef struct xbfs_comm xbfs_comm;
 
-/* Build rank `rank`'s partition.  Every rank passes the SAME full tuple list
- * (src, dst: num_edges ids of width opts->id_bytes, host or device per opts);
- * the rank keeps the arcs whose source it owns (both directions of every tuple,
- * self-loops and duplicates dropped, rows id-sorted) and re-arranges its rows by
- * neighbour degree, descending, where the degree of a remote
- * neighbour is its tuple-incidence count (reading R-6 in DESIGN.md).
- * Errors: INVALID_ARG (nranks outside [1, XBFS_DIST_MAX_RANKS], rank outside
- * [0, nranks), plus xbfs_build_csr's), OUT_OF_MEMORY, CUDA. */
-xbfs_status xbfs_dist_build(const void* src, const void* dst, int64_t num_edges, int64_t num_vertices,
-                            int32_t nranks, int32_t rank, const xbfs_build_opts* opts, xbfs_dist** out);
+/* Local.  A fresh communicator id (128 bytes, the analogue of an ncclUniqueId):
+ * rank 0 calls it and broadcasts the bytes to the other ranks (torch.distributed).
+ * Errors: INVALID_ARG (NULL). */
+xbfs_status xbfs_get_unique_id(uint8_t id[XBFS_UNIQUE_ID_BYTES]);
 
-/* Owned range and sizes.  Any out pointer may be NULL. */
-xbfs_status xbfs_dist_info(const xbfs_dist* d, int64_t* first, int64_t* count, int64_t* local_arcs,
-                           int64_t* num_vertices);
+/* Collective over the nranks processes of one node.  rank 0 creates the shared
+ * segment named in `id`, the others attach to it (waiting up to 600 s).  Makes
+ * no CUDA call.  Errors: INVALID_ARG (NULL, not an xbfs id, rank outside
+ * [0, nranks), nranks outside [1, XBFS_DIST_MAX_RANKS], nranks differing from
+ * rank 0's), STATE (segment could not be created / a peer never arrived). */
+xbfs_status xbfs_comm_init(const uint8_t id[XBFS_UNIQUE_ID_BYTES], int32_t nranks, int32_t rank, xbfs_comm** out);
 
-/* IPC handle (XBFS_IPC_HANDLE_BYTES bytes) of this rank's shared region (the
- * three frontier replicas + the inbox); exchange it with every rank. */
-xbfs_status xbfs_dist_export(xbfs_dist* d, void* handle_out);
+/* Collective host-side barrier and int64 sum all-reduce (count <= 512) of the
+ * communicator (used inside xbfs_run_dist; exported for the caller's harness and
+ * the CPU tests).  Errors: INVALID_ARG, STATE (a peer did not arrive in 600 s). */
+xbfs_status xbfs_comm_barrier(xbfs_comm* c);
+xbfs_status xbfs_comm_allreduce_i64(xbfs_comm* c, const int64_t* in, int64_t* out, int32_t count);
 
-/* Map the peers' shared regions.  handles: nranks * XBFS_IPC_HANDLE_BYTES in
- * rank order (this rank's own entry is ignored).  Call once, after every rank
- * exported; peers may be other GPUs (NVLink P2P) or the same GPU (tests). */
-xbfs_status xbfs_dist_attach(xbfs_dist* d, const void* handles);
+/* Collective.  Build this rank's partition from ITS OWN share of the input tuples:
+ * src/dst hold local_edges ids (width opts->id_bytes; host or device per opts),
+ * any split of the M tuples over the ranks (e.g. rank r generates tuples
+ * [r*M/p, (r+1)*M/p)).  The library ships every arc (both directions of each
+ * tuple) to the owner of its source over peer memory (counts all-gathered first),
+ * then each owner sorts, drops self-loops and duplicates (C-3), builds its rows
+ * and records per-vertex tuple counts (Graph500 m, O-6); the owned degrees are
+ * all-gathered and every row is re-arranged as xbfs_reorder mode 1 does.  The
+ * handle runs only with xbfs_run_dist and is freed with xbfs_destroy (local).
+ * opts->directed is unsupported (UNSUPPORTED).  Errors: INVALID_ARG (NULL, N out
+ * of (0, 2^31), ids >= N on any rank), OUT_OF_MEMORY, CUDA, STATE (comm). */
+xbfs_status xbfs_build_csr_dist(xbfs_comm* c, const void* src, const void* dst, int64_t local_edges,
+                                int64_t num_vertices, const xbfs_build_opts* opts, xbfs_graph** out);
 
-/* Start a BFS from global vertex `source`: resets this rank's state and writes
- * every element of the caller-owned DEVICE arrays level_local[count] and
- * parent_local[count] (parent values are global ids).  counts[] receives this
- * rank's {owns source, deg(source), tuples of source, non-isolated owned
- * vertices, local arcs, 0, 0, 0}; all-reduce them (sum) and pass the result to
- * xbfs_dist_advance, which also acts as the barrier before the first level. */
-xbfs_status xbfs_dist_begin(xbfs_dist* d, int64_t source, int32_t* level_local, int32_t* parent_local,
-                            const xbfs_run_opts* opts, int64_t counts[XBFS_DIST_NCOUNTS]);
+/* Local.  This rank's owned vertex range [*first, *first + *count). */
+xbfs_status xbfs_partition_range(const xbfs_graph* g, int64_t* first, int64_t* count);
 
-/* Run phase 0 or 1 of the current level on this rank and synchronise its
- * stream.  After the level's last phase (phase 0 for BU, phase 1 for TD)
- * counts[] = this rank's {new frontier vertices, their degree sum, their tuple
- * count (Graph500 m), arcs probed by BU, 0...}; zeros otherwise.  A caller
- * barrier must separate phase 0 and phase 1 of a TD level; the all-reduce of
- * the counts separates levels. */
-xbfs_status xbfs_dist_level(xbfs_dist* d, int32_t phase, int64_t counts[XBFS_DIST_NCOUNTS]);
+/* Collective.  One BFS from global vertex `source`, every level of it:
+ * writes every element of the caller-owned DEVICE arrays level_local[count] and
+ * parent_local[count] (parent values are global ids; -1 if unreached; semantics
+ * of xbfs_run).  opts: strategy parameters as xbfs_run (driver, plan, small_edges,
+ * lookahead are ignored).  stats (may be NULL; then the call still synchronises,
+ * as the level loop is host-driven): elapsed_ms = this rank's device time from
+ * init to the end of the last level (CUDA events; take the max over ranks),
+ * num_levels, vertices_reached, arcs_traversed, input_edges_traversed = GLOBAL
+ * values, and the per-level arrays (strategy, frontier_vertices, frontier_edges,
+ * unvisited, bu_probes) of global counts.  Errors: INVALID_ARG (source outside
+ * [0, N), NULL outputs with count > 0), STATE, CUDA. */
+xbfs_status xbfs_run_dist(xbfs_graph* g, int64_t source, int32_t* level_local, int32_t* parent_local,
+                          const xbfs_run_opts* opts, xbfs_run_stats* stats);
 
-/* Apply the all-reduced counters (identical on every rank) and choose the next
- * level's strategy.  *done = 1 when the next frontier is empty. */
-xbfs_status xbfs_dist_advance(xbfs_dist* d, const int64_t global_counts[XBFS_DIST_NCOUNTS],
-                              int32_t* strategy_out, int32_t* done);
-
-/* Per-level log of the last BFS (host arrays of cap entries, NULL to skip);
- * *num_levels = number of levels, *input_edges = Graph500 m (O-6) over all
- * ranks.  Any out pointer may be NULL. */
-xbfs_status xbfs_dist_levels(const xbfs_dist* d, int32_t cap, int8_t* strategy, int64_t* frontier_vertices,
-                             int64_t* frontier_edges, int32_t* num_levels, int64_t* input_edges);
-
-/* NULL-safe. */
-void xbfs_dist_destroy(xbfs_dist* d);
+/* Local.  Frees the communicator (NULL-safe); destroy the graphs built on it first. */
+void xbfs_comm_destroy(xbfs_comm* c);
 
 #ifdef __cplusplus
 }

@@ -103,6 +103,7 @@ xbfs_status xbfs_copy_csr(const xbfs_graph* gc, int64_t* row_ptr_host, int32_t* 
     if (!g || !row_ptr_host || (!col_host && g->arcs > 0))
         return xbfs::set_error(XBFS_ERR_INVALID_ARG, "xbfs_copy_csr: NULL argument");
     if (g->poisoned) return xbfs::set_error(XBFS_ERR_STATE, "handle poisoned by an earlier failure");
+    if (g->dist) return xbfs::set_error(XBFS_ERR_STATE, "xbfs_copy_csr: distributed handle");
     XBFS_CUDA(g, cudaSetDevice(g->device));
     XBFS_CUDA(g, cudaMemcpyAsync(row_ptr_host, g->row_ptr, (g->n + 1) * sizeof(long long),
                                  cudaMemcpyDeviceToHost, g->stream));
@@ -118,6 +119,7 @@ void xbfs_destroy(xbfs_graph* g) {
     cudaSetDevice(g->device);
     if (g->stream) cudaStreamSynchronize(g->stream);
     if (g->copy_stream) cudaStreamSynchronize(g->copy_stream);
+    if (g->dist) xbfs::dist_destroy(g->dist);
     if (g->loop_exec) cudaGraphExecDestroy(g->loop_exec);
     void* dev[] = {g->row_ptr, g->col, g->tcount, g->nonisolated, g->visited, g->fb, g->qv,
                    g->qoff, g->qdelta, g->tile_first, g->st, g->log, g->red_scratch,

@@ -460,6 +460,7 @@ extern "C" xbfs_status xbfs_reorder(xbfs_graph* g, int32_t mode) {
     if (!g) return set_error(XBFS_ERR_INVALID_ARG, "xbfs_reorder: NULL handle");
     if (mode != 0 && mode != 1) return set_error(XBFS_ERR_INVALID_ARG, "xbfs_reorder: mode must be 0 or 1");
     if (g->poisoned) return set_error(XBFS_ERR_STATE, "handle poisoned by an earlier failure");
+    if (g->dist) return set_error(XBFS_ERR_STATE, "xbfs_reorder: a distributed handle is re-arranged at build time");
     if (g->arcs == 0) { g->reorder_mode = mode; return XBFS_OK; }
     XBFS_CUDA(g, cudaSetDevice(g->device));
     const long long n = g->n;

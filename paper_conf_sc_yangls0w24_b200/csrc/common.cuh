@@ -186,9 +186,18 @@ struct xbfs_graph {
     xbfs::KArgs kargs() const;
 };
 
+struct xbfs_comm;
 namespace xbfs {
 // driver state created at build / re-arrangement time (bfs.cu)
 xbfs_status prepare_drivers(xbfs_graph* g);
+// multi-GPU (comm.cu host collectives; dist.cu partition)
+constexpr int kMaxCommRanks = 16;
+xbfs_status comm_barrier(xbfs_comm* c);
+xbfs_status comm_allgather(xbfs_comm* c, const void* mine, size_t bytes, void* all);
+xbfs_status comm_allreduce_sum(xbfs_comm* c, const int64_t* in, int64_t* out, int n);
+int comm_rank(const xbfs_comm* c);
+int comm_size(const xbfs_comm* c);
+void dist_destroy(struct xbfs_dist_part* d);
 // error plumbing (api.cu)
 xbfs_status set_error(xbfs_status s, const char* fmt, ...);
 xbfs_status cuda_fail(xbfs_graph* g, cudaError_t e, const char* what);

@@ -1,6 +1,8 @@
 // dist.cu — multi-GPU XBFS (include/xbfs_dist.h): 1D vertex partition, one
-// process per GPU, frontier exchange fused into the producing kernels as stores
-// to peer memory (CUDA IPC; NVLink/NVSwitch between GPUs).
+// process per GPU, the frontier exchange fused into the producing kernels as
+// stores to peer memory (CUDA IPC; NVLink/NVSwitch between GPUs), the level loop
+// and the per-level counter all-reduce inside xbfs_run_dist (comm.cu's host
+// collectives; reading R-10).
 //
 // Per rank: owned rows [lo, lo+count) with global neighbour ids, a local visited
 // bitmap over the owned range, three replicated N-bit frontier bitmaps and an
@@ -17,12 +19,20 @@
 #include "common.cuh"
 #include "xbfs_dist.h"
 
+#define XBFS_TRY_D(expr)                        \
+    do {                                        \
+        xbfs_status _s = (expr);                \
+        if (_s != XBFS_OK) return _s;           \
+    } while (0)
+
 namespace xbfs {
 namespace dist {
 
 constexpr unsigned FULL = 0xffffffffu;
 constexpr int kB = 256;
 constexpr int kChunkArcs = 1024;     // TD work item: one vertex, up to 1024 arcs
+constexpr unsigned long long kFirst = 1ull << 63;   // build key flag: the tuple's first endpoint is the row
+constexpr unsigned long long kDrop = ~0ull;         // build key of a self-loop (sorted last, dropped)
 
 struct DAcc {
     unsigned long long found, edges, m, probes;
@@ -71,12 +81,6 @@ __global__ void k_seed(DArgs a, long long s) {
         a.parent[vl] = (int)s;
         a.vis[vl >> 5] |= 1u << (vl & 31);
     }
-}
-
-__global__ __launch_bounds__(kB) void k_clear(unsigned* bm, long long words) {
-    for (long long w = blockIdx.x * (long long)blockDim.x + threadIdx.x; w < words;
-         w += (long long)gridDim.x * blockDim.x)
-        bm[w] = 0;
 }
 
 // Store one owned word of F_{k+1} into every replica (local + peers): the
@@ -228,8 +232,8 @@ __global__ __launch_bounds__(kB) void k_td(DArgs a, int k) {
 }
 
 // TD phase 1: inbox ∧ ¬visited are new owned frontier vertices; each finds its
-// parent with a bottom-up probe against F_k, then the owned F_{k+1} words go to
-// every replica and are counted.
+// parent with a bottom-up probe against F_k (the first vertex of its row in F_k),
+// then the owned F_{k+1} words go to every replica and are counted.
 __global__ __launch_bounds__(kB) void k_merge(DArgs a, int k) {
     const unsigned* cur = a.fb[k % 3];
     const int slot = (k + 1) % 3;
@@ -273,23 +277,55 @@ __global__ __launch_bounds__(kB) void k_merge(DArgs a, int k) {
 }
 
 // ---------------------------------------------------------------- build
-template <typename IdT>
-__global__ __launch_bounds__(kB) void k_pack_owned(const IdT* __restrict__ src, const IdT* __restrict__ dst,
-                                                   long long m, long long n, long long lo, long long count, int nb,
-                                                   unsigned long long* __restrict__ keys,
-                                                   unsigned long long* __restrict__ nkeys, int* __restrict__ inc,
-                                                   int* __restrict__ tcount, int* __restrict__ bad) {
+// Pass 1 over this rank's tuples: per destination rank, how many arc keys go
+// there (both directions of every tuple; a self-loop only once, for its tuple
+// count).  Pass 2 writes the keys (row_local << nb | neighbour, kFirst on the
+// tuple's first endpoint: tcount) into the destination's segment of the send
+// buffer.  Ids out of range set *bad.
+template <typename IdT, bool WRITE>
+__global__ __launch_bounds__(kB) void k_route(const IdT* __restrict__ src, const IdT* __restrict__ dst, long long m,
+                                              long long n, long long blk, int nb,
+                                              unsigned long long* __restrict__ cursor,
+                                              unsigned long long* __restrict__ keys, int* __restrict__ bad) {
+    __shared__ unsigned long long s_cnt[XBFS_DIST_MAX_RANKS];
+    if (!WRITE) {
+        if (threadIdx.x < XBFS_DIST_MAX_RANKS) s_cnt[threadIdx.x] = 0;
+        __syncthreads();
+    }
     for (long long e = blockIdx.x * (long long)blockDim.x + threadIdx.x; e < m;
          e += (long long)gridDim.x * blockDim.x) {
         const long long u = (long long)src[e], v = (long long)dst[e];
         if (u < 0 || v < 0 || u >= n || v >= n) { *bad = 1; continue; }
-        const bool ou = u >= lo && u < lo + count, ov = v >= lo && v < lo + count;
-        if (ou) atomicAdd(&tcount[u - lo], 1);
-        if (u == v) continue;
-        atomicAdd(&inc[u], 1);
-        atomicAdd(&inc[v], 1);
-        if (ou) keys[atomicAdd(nkeys, 1ull)] = ((unsigned long long)(u - lo) << nb) | (unsigned long long)v;
-        if (ov) keys[atomicAdd(nkeys, 1ull)] = ((unsigned long long)(v - lo) << nb) | (unsigned long long)u;
+        const int ou = (int)(u / blk), ov = (int)(v / blk);
+        if (!WRITE) {
+            atomicAdd(&s_cnt[ou], 1ull);
+            if (u != v) atomicAdd(&s_cnt[ov], 1ull);
+        } else {
+            keys[atomicAdd(&cursor[ou], 1ull)] =
+                kFirst | ((unsigned long long)(u - (long long)ou * blk) << nb) | (unsigned long long)v;
+            if (u != v)
+                keys[atomicAdd(&cursor[ov], 1ull)] = ((unsigned long long)(v - (long long)ov * blk) << nb) |
+                                                     (unsigned long long)u;
+        }
+    }
+    if (!WRITE) {
+        __syncthreads();
+        if (threadIdx.x < XBFS_DIST_MAX_RANKS && s_cnt[threadIdx.x]) atomicAdd(&cursor[threadIdx.x], s_cnt[threadIdx.x]);
+    }
+}
+
+// Received keys: count the tuples of every owned first endpoint (Graph500 m,
+// O-6: duplicates and self-loops included), clear the flag, drop self-loops.
+__global__ __launch_bounds__(kB) void k_strip(unsigned long long* __restrict__ keys, long long nk, long long lo, int nb,
+                                              int* __restrict__ tcount) {
+    const unsigned long long lowmask = (1ull << nb) - 1ull;
+    for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < nk;
+         i += (long long)gridDim.x * blockDim.x) {
+        unsigned long long key = keys[i];
+        const long long row = (long long)((key & ~kFirst) >> nb);
+        if (key & kFirst) atomicAdd(&tcount[row], 1);
+        key &= ~kFirst;
+        keys[i] = ((long long)(key & lowmask) == lo + row) ? kDrop : key;
     }
 }
 
@@ -315,10 +351,24 @@ __global__ __launch_bounds__(kB) void k_fill64(long long* p, long long n, long l
         p[i] = v;
 }
 
-// Reorder keys: (row << db) | (maxinc - inc[col]); stable, so ties stay id-ascending.
+__global__ __launch_bounds__(kB) void k_degrees(const long long* __restrict__ row_ptr, long long count,
+                                                int* __restrict__ deg, unsigned* __restrict__ maxdeg) {
+    unsigned mx = 0;
+    for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < count;
+         v += (long long)gridDim.x * blockDim.x) {
+        const int d = (int)(row_ptr[v + 1] - row_ptr[v]);
+        deg[v] = d;
+        mx = max(mx, (unsigned)d);
+    }
+    for (int o = 16; o; o >>= 1) mx = max(mx, __shfl_xor_sync(FULL, mx, o));
+    if ((threadIdx.x & 31) == 0 && mx) atomicMax(maxdeg, mx);
+}
+
+// Re-arrangement keys: (row << db) | (maxdeg - deg[col]); stable, so ties stay
+// id-ascending: exactly xbfs_reorder's order (C-12) with true degrees.
 __global__ __launch_bounds__(kB) void k_rkeys(const long long* __restrict__ row_ptr, const int* __restrict__ col,
-                                              const int* __restrict__ inc, long long count, long long a, int db,
-                                              unsigned long long maxinc, unsigned long long* __restrict__ keys) {
+                                              const int* __restrict__ deg_all, long long count, long long a, int db,
+                                              unsigned long long maxdeg, unsigned long long* __restrict__ keys) {
     for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < a;
          i += (long long)gridDim.x * blockDim.x) {
         long long lo = 0, hi = count - 1;
@@ -326,7 +376,7 @@ __global__ __launch_bounds__(kB) void k_rkeys(const long long* __restrict__ row_
             const long long mid = (lo + hi + 1) >> 1;
             if (row_ptr[mid] <= i) lo = mid; else hi = mid - 1;
         }
-        keys[i] = ((unsigned long long)lo << db) | (maxinc - (unsigned long long)inc[col[i]]);
+        keys[i] = ((unsigned long long)lo << db) | (maxdeg - (unsigned long long)deg_all[col[i]]);
     }
 }
 
@@ -352,15 +402,6 @@ __global__ __launch_bounds__(kB) void k_facts(const long long* __restrict__ row_
     if ((threadIdx.x & 31) == 0 && c) atomicAdd(nnon, c);
 }
 
-__global__ __launch_bounds__(kB) void k_maxinc(const int* __restrict__ inc, long long n, unsigned* out) {
-    unsigned mx = 0;
-    for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n;
-         i += (long long)gridDim.x * blockDim.x)
-        mx = max(mx, (unsigned)inc[i]);
-    for (int o = 16; o; o >>= 1) mx = max(mx, __shfl_xor_sync(FULL, mx, o));
-    if ((threadIdx.x & 31) == 0) atomicMax(out, mx);
-}
-
 inline int grid_for(long long n, int cap = 148 * 16) {
     long long g = (n + kB - 1) / kB;
     return (int)std::max(1ll, std::min<long long>(g, cap));
@@ -368,19 +409,30 @@ inline int grid_for(long long n, int cap = 148 * 16) {
 
 inline int bitlen(unsigned long long x) { return x ? 64 - __builtin_clzll(x) : 0; }
 
+// host mirror of choose_strategy (bfs.cu): identical inputs on every rank
+int choose(const xbfs_run_opts& o, long long arcs, long long fsize, long long fprev, long long fedges,
+           long long unvisited, int prev) {
+    if (o.force_strategy >= 0) return o.force_strategy;
+    const double e = (double)fedges, A = (double)arcs;
+    if (arcs > 0 && e > o.alpha * A) return XBFS_BU;                                          // P:L87, C-8
+    if (o.bu_stay > 0.0 && prev == XBFS_BU && (double)unvisited * o.bu_stay < e) return XBFS_BU;   // C-11
+    if ((double)fsize > o.grow * (double)fprev && arcs > 0 && e > o.ratio_min * A) return XBFS_SS; // C-10
+    return XBFS_SF;
+}
+
 }  // namespace dist
 }  // namespace xbfs
 
 using namespace xbfs;
 using namespace xbfs::dist;
 
-struct xbfs_dist {
-    int device = 0;
-    cudaStream_t stream = nullptr;
-    bool poisoned = false;
+// The multi-GPU part of a graph handle (xbfs_graph::dist).
+struct xbfs_dist_part {
+    xbfs_comm* comm = nullptr;
     int rank = 0, nranks = 1;
-    long long n = 0, lo = 0, count = 0, blk = 0, arcs = 0, fwords = 0, fwords_pad = 0, cw = 0, blk_w = 0;
-    long long nonisolated_local = 0;
+    long long n = 0, lo = 0, count = 0, blk = 0, arcs_local = 0, arcs_global = 0, fwords = 0, fwords_pad = 0,
+              cw = 0, blk_w = 0;
+    long long nonisolated_local = 0, nonisolated_global = 0;
     long long* row_ptr = nullptr;
     int* col = nullptr;
     unsigned long long* head = nullptr;
@@ -392,20 +444,12 @@ struct xbfs_dist {
     unsigned long long* items = nullptr;
     long long items_cap = 0;
     DAcc* acc = nullptr;
-    DAcc* acc_host = nullptr;
-    bool attached = false;
-    // current BFS
-    int* level = nullptr;
-    int* parent = nullptr;
-    int k = 0, strategy = 0, started = 0;
-    long long fsize = 0, fedges = 0, fprev = 0, unvisited = 0, m_total = 0, arcs_global = 0;
-    xbfs_run_opts opts;
-    std::vector<int8_t> log_s;
-    std::vector<long long> log_f, log_e;
+    DAcc* acc_host = nullptr;               // pinned
+    cudaEvent_t ev0 = nullptr, ev1 = nullptr;
 
     unsigned* fb_of(unsigned* base, int i) const { return base + (long long)i * fwords_pad; }
     unsigned* inbox_of(unsigned* base) const { return base + 3 * fwords_pad; }
-    DArgs args() const {
+    DArgs args(int* level, int* parent) const {
         DArgs a;
         a.row_ptr = row_ptr;
         a.col = col;
@@ -438,191 +482,315 @@ struct xbfs_dist {
     }
 };
 
+namespace xbfs {
+void dist_destroy(xbfs_dist_part* d) {
+    if (!d) return;
+    for (int p = 0; p < XBFS_DIST_MAX_RANKS; ++p)
+        if (d->peer_base[p]) cudaIpcCloseMemHandle(d->peer_base[p]);
+    void* ptrs[] = {d->row_ptr, d->col, d->head, d->tcount, d->noniso, d->vis, d->shared, d->items, d->acc};
+    for (void* p : ptrs)
+        if (p) cudaFree(p);
+    if (d->acc_host) cudaFreeHost(d->acc_host);
+    if (d->ev0) cudaEventDestroy(d->ev0);
+    if (d->ev1) cudaEventDestroy(d->ev1);
+    delete d;
+}
+}  // namespace xbfs
+
 namespace {
 
-xbfs_status dfail(xbfs_dist* d, cudaError_t e, const char* what) {
-    if (d) d->poisoned = true;
-    return cuda_fail(nullptr, e, what);
+#define DCUDA(g, call) XBFS_CUDA(g, call)
+#define DTRY(expr) XBFS_TRY_D(expr)
+
+// A device buffer every rank can see: allocate locally, all-gather the IPC
+// handles, open the peers' (peer memory; the same device in the tests).
+xbfs_status exchange_handles(xbfs_graph* g, xbfs_comm* c, void* mine, void** peers) {
+    const int nr = comm_size(c), r = comm_rank(c);
+    if (nr == 1) {
+        peers[0] = mine;
+        return XBFS_OK;
+    }
+    cudaIpcMemHandle_t h;
+    memset(&h, 0, sizeof(h));
+    if (mine) DCUDA(g, cudaIpcGetMemHandle(&h, mine));
+    std::vector<cudaIpcMemHandle_t> all(nr);
+    DTRY(comm_allgather(c, &h, sizeof(h), all.data()));
+    for (int p = 0; p < nr; ++p) {
+        peers[p] = nullptr;
+        if (p == r) { peers[p] = mine; continue; }
+        cudaIpcMemHandle_t z;
+        memset(&z, 0, sizeof(z));
+        if (!memcmp(&all[p], &z, sizeof(z))) continue;   // that rank had nothing to share
+        DCUDA(g, cudaIpcOpenMemHandle(&peers[p], all[p], cudaIpcMemLazyEnablePeerAccess));
+    }
+    return XBFS_OK;
 }
 
-#define DCUDA(d, call)                                              \
-    do {                                                            \
-        cudaError_t _e = (call);                                    \
-        if (_e != cudaSuccess) return dfail((d), _e, #call);        \
-    } while (0)
-
-// host mirror of choose_strategy (bfs.cu): identical inputs on every rank
-int choose(const xbfs_run_opts& o, long long arcs, long long fsize, long long fprev, long long fedges,
-           long long unvisited, int prev) {
-    if (o.force_strategy >= 0) return o.force_strategy;
-    const double ratio = arcs > 0 ? (double)fedges / (double)arcs : 0.0;
-    if (ratio > o.alpha) return XBFS_BU;
-    if (o.bu_stay > 0.0 && prev == XBFS_BU && (double)unvisited * o.bu_stay < (double)fedges) return XBFS_BU;
-    if ((double)fsize > o.grow * (double)fprev && ratio > o.ratio_min) return XBFS_SS;
-    return XBFS_SF;
+void close_handles(xbfs_comm* c, void** peers) {
+    for (int p = 0; p < comm_size(c); ++p)
+        if (p != comm_rank(c) && peers[p]) cudaIpcCloseMemHandle(peers[p]);
 }
 
 template <typename IdT>
-xbfs_status pack(xbfs_dist* d, const void* src, const void* dst, long long m, bool on_dev, int nb,
-                 unsigned long long* keys, unsigned long long* nkeys, int* inc, int* bad) {
+xbfs_status route(xbfs_graph* g, xbfs_dist_part* d, const void* src, const void* dst, long long m, bool on_dev, int nb,
+                  unsigned long long* cursor, unsigned long long* keys, int* bad, bool write) {
     const IdT* s = (const IdT*)src;
     const IdT* t = (const IdT*)dst;
     IdT *ds = nullptr, *dd = nullptr;
     const long long chunk = on_dev ? std::max(m, 1ll) : std::min<long long>(std::max(m, 1ll), 1ll << 27);
     if (!on_dev && m > 0) {
-        DCUDA(d, cudaMalloc(&ds, chunk * sizeof(IdT)));
-        DCUDA(d, cudaMalloc(&dd, chunk * sizeof(IdT)));
+        DCUDA(g, cudaMalloc(&ds, chunk * sizeof(IdT)));
+        DCUDA(g, cudaMalloc(&dd, chunk * sizeof(IdT)));
     }
-    for (long long e0 = 0; e0 < m; e0 += chunk) {
-        const long long c = std::min(chunk, m - e0);
+    xbfs_status st = XBFS_OK;
+    for (long long e0 = 0; e0 < m && st == XBFS_OK; e0 += chunk) {
+        const long long cn = std::min(chunk, m - e0);
         const IdT* ps = s + e0;
         const IdT* pt = t + e0;
         if (!on_dev) {
-            DCUDA(d, cudaMemcpyAsync(ds, ps, c * sizeof(IdT), cudaMemcpyHostToDevice, d->stream));
-            DCUDA(d, cudaMemcpyAsync(dd, pt, c * sizeof(IdT), cudaMemcpyHostToDevice, d->stream));
+            cudaMemcpyAsync(ds, ps, cn * sizeof(IdT), cudaMemcpyHostToDevice, g->stream);
+            cudaMemcpyAsync(dd, pt, cn * sizeof(IdT), cudaMemcpyHostToDevice, g->stream);
             ps = ds;
             pt = dd;
         }
-        k_pack_owned<IdT><<<grid_for(c), kB, 0, d->stream>>>(ps, pt, c, d->n, d->lo, d->count, nb, keys, nkeys,
-                                                            inc, d->tcount, bad);
-        DCUDA(d, cudaGetLastError());
+        if (write)
+            k_route<IdT, true><<<grid_for(cn), kB, 0, g->stream>>>(ps, pt, cn, d->n, d->blk, nb, cursor, keys, bad);
+        else
+            k_route<IdT, false><<<grid_for(cn), kB, 0, g->stream>>>(ps, pt, cn, d->n, d->blk, nb, cursor, keys, bad);
+        const cudaError_t e = cudaGetLastError();
+        if (e != cudaSuccess) st = cuda_fail(g, e, "k_route");
     }
-    DCUDA(d, cudaStreamSynchronize(d->stream));
+    if (st == XBFS_OK) {
+        const cudaError_t e = cudaStreamSynchronize(g->stream);
+        if (e != cudaSuccess) st = cuda_fail(g, e, "k_route sync");
+    }
     if (ds) { cudaFree(ds); cudaFree(dd); }
-    return XBFS_OK;
+    return st;
 }
 
-xbfs_status build_impl(xbfs_dist* d, const void* src, const void* dst, long long m, const xbfs_build_opts& o) {
+xbfs_status build_dist(xbfs_graph* g, xbfs_dist_part* d, const void* src, const void* dst, long long m,
+                       const xbfs_build_opts& o) {
+    xbfs_comm* c = d->comm;
+    const int nr = d->nranks, me = d->rank;
     const long long n = d->n, count = d->count;
-    const int nb_row = std::max(1, bitlen((unsigned long long)std::max(count - 1, 1ll)));
+    const int nb_row = std::max(1, bitlen((unsigned long long)std::max(d->blk - 1, 1ll)));
     const int nb = std::max(1, bitlen((unsigned long long)(n - 1)));
-    if (nb_row + nb > 64) return set_error(XBFS_ERR_UNSUPPORTED, "dist key does not fit in 64 bits");
-    int* inc = nullptr;
-    int* bad = nullptr;
-    unsigned long long *k0 = nullptr, *k1 = nullptr, *nkeys = nullptr;
-    DCUDA(d, cudaMalloc(&inc, n * sizeof(int)));
-    DCUDA(d, cudaMemsetAsync(inc, 0, n * sizeof(int), d->stream));
-    DCUDA(d, cudaMalloc(&d->tcount, std::max(count, 1ll) * sizeof(int)));
-    DCUDA(d, cudaMemsetAsync(d->tcount, 0, std::max(count, 1ll) * sizeof(int), d->stream));
-    DCUDA(d, cudaMalloc(&bad, sizeof(int)));
-    DCUDA(d, cudaMemsetAsync(bad, 0, sizeof(int), d->stream));
-    DCUDA(d, cudaMalloc(&nkeys, sizeof(unsigned long long)));
-    DCUDA(d, cudaMemsetAsync(nkeys, 0, sizeof(unsigned long long), d->stream));
-    // upper bound on owned arcs: 2 per tuple
-    const long long cap = std::max(2 * m, 1ll);
-    DCUDA(d, cudaMalloc(&k0, cap * sizeof(unsigned long long)));
+    if (nb_row + nb > 63) return set_error(XBFS_ERR_UNSUPPORTED, "dist key does not fit in 63 bits");
     const bool on_dev = o.edges_on_device != 0;
-    xbfs_status st = o.id_bytes == 8 ? pack<long long>(d, src, dst, m, on_dev, nb, k0, nkeys, inc, bad)
-                                     : pack<unsigned int>(d, src, dst, m, on_dev, nb, k0, nkeys, inc, bad);
-    if (st != XBFS_OK) return st;
-    int hbad = 0;
-    unsigned long long hk = 0;
-    DCUDA(d, cudaMemcpy(&hbad, bad, sizeof(int), cudaMemcpyDeviceToHost));
-    DCUDA(d, cudaMemcpy(&hk, nkeys, sizeof(hk), cudaMemcpyDeviceToHost));
-    if (hbad) {
-        cudaFree(inc); cudaFree(bad); cudaFree(k0); cudaFree(nkeys);
-        return set_error(XBFS_ERR_INVALID_ARG, "edge id out of range [0, %lld)", n);
+    // 1. how many keys go to every rank (pass 1), all-gathered: row r = what rank r sends
+    unsigned long long *cursor = nullptr, *sendk = nullptr;
+    int* bad = nullptr;
+    DCUDA(g, cudaMalloc(&cursor, XBFS_DIST_MAX_RANKS * sizeof(unsigned long long)));
+    DCUDA(g, cudaMemsetAsync(cursor, 0, XBFS_DIST_MAX_RANKS * sizeof(unsigned long long), g->stream));
+    DCUDA(g, cudaMalloc(&bad, sizeof(int)));
+    DCUDA(g, cudaMemsetAsync(bad, 0, sizeof(int), g->stream));
+    DTRY(o.id_bytes == 8 ? route<long long>(g, d, src, dst, m, on_dev, nb, cursor, nullptr, bad, false)
+                         : route<unsigned>(g, d, src, dst, m, on_dev, nb, cursor, nullptr, bad, false));
+    long long mine[XBFS_DIST_MAX_RANKS + 1] = {0};
+    {
+        unsigned long long hc[XBFS_DIST_MAX_RANKS];
+        int hbad = 0;
+        DCUDA(g, cudaMemcpy(hc, cursor, sizeof(hc), cudaMemcpyDeviceToHost));
+        DCUDA(g, cudaMemcpy(&hbad, bad, sizeof(int), cudaMemcpyDeviceToHost));
+        for (int p = 0; p < nr; ++p) mine[p] = (long long)hc[p];
+        mine[XBFS_DIST_MAX_RANKS] = hbad;
     }
-    long long nk = (long long)hk;
-    DCUDA(d, cudaMalloc(&k1, std::max(nk, 1ll) * sizeof(unsigned long long)));
+    std::vector<long long> cnt((size_t)nr * (XBFS_DIST_MAX_RANKS + 1));
+    DTRY(comm_allgather(c, mine, sizeof(mine), cnt.data()));
+    auto C = [&](int from, int to) { return cnt[(size_t)from * (XBFS_DIST_MAX_RANKS + 1) + to]; };
+    for (int p = 0; p < nr; ++p)
+        if (C(p, XBFS_DIST_MAX_RANKS)) {
+            cudaFree(cursor); cudaFree(bad);
+            return set_error(XBFS_ERR_INVALID_ARG, "edge id out of range [0, %lld) on rank %d", n, p);
+        }
+    long long send_total = 0, recv_total = 0;
+    for (int p = 0; p < nr; ++p) { send_total += C(me, p); recv_total += C(p, me); }
+    // 2. keys into per-destination segments of the send buffer (pass 2)
+    std::vector<unsigned long long> start(XBFS_DIST_MAX_RANKS, 0);
+    for (int p = 1; p < nr; ++p) start[p] = start[p - 1] + (unsigned long long)C(me, p - 1);
+    DCUDA(g, cudaMemcpy(cursor, start.data(), XBFS_DIST_MAX_RANKS * sizeof(unsigned long long), cudaMemcpyHostToDevice));
+    DCUDA(g, cudaMalloc(&sendk, std::max(send_total, 1ll) * sizeof(unsigned long long)));
+    DTRY(o.id_bytes == 8 ? route<long long>(g, d, src, dst, m, on_dev, nb, cursor, sendk, bad, true)
+                         : route<unsigned>(g, d, src, dst, m, on_dev, nb, cursor, sendk, bad, true));
+    cudaFree(cursor);
+    cudaFree(bad);
+    // 3. ship every segment to its owner over peer memory: rank p's keys for me land at
+    //    offset sum_{q<p} C(q, me) of my receive buffer (one rank: the send buffer is it)
+    unsigned long long* recvk = nullptr;
+    long long nk = recv_total;
+    if (nr == 1) {
+        recvk = sendk;
+        sendk = nullptr;
+    } else {
+        DCUDA(g, cudaMalloc(&recvk, std::max(recv_total, 1ll) * sizeof(unsigned long long)));
+        void* peers[XBFS_DIST_MAX_RANKS];
+        DTRY(exchange_handles(g, c, recvk, peers));
+        for (int p = 0; p < nr; ++p) {
+            long long off = 0;
+            for (int q = 0; q < me; ++q) off += C(q, p);
+            if (C(me, p) == 0) continue;
+            DCUDA(g, cudaMemcpyAsync((unsigned long long*)peers[p] + off, sendk + start[p],
+                                     C(me, p) * sizeof(unsigned long long), cudaMemcpyDefault, g->stream));
+        }
+        DCUDA(g, cudaStreamSynchronize(g->stream));
+        DTRY(comm_barrier(c));                  // every segment has landed everywhere
+        close_handles(c, peers);
+        cudaFree(sendk);
+        sendk = nullptr;
+        DTRY(comm_barrier(c));                  // nobody frees a buffer a peer still maps
+    }
+    // 4. tuple counts, self-loops dropped, sort, dedup (C-3), rows
+    DCUDA(g, cudaMalloc(&d->tcount, std::max(count, 1ll) * sizeof(int)));
+    DCUDA(g, cudaMemsetAsync(d->tcount, 0, std::max(count, 1ll) * sizeof(int), g->stream));
+    DCUDA(g, cudaMalloc(&d->row_ptr, (count + 1) * sizeof(long long)));
     long long arcs = 0;
-    d->row_ptr = nullptr;
-    DCUDA(d, cudaMalloc(&d->row_ptr, (count + 1) * sizeof(long long)));
     if (nk > 0) {
-        cub::DoubleBuffer<unsigned long long> db(k0, k1);
+        k_strip<<<grid_for(nk), kB, 0, g->stream>>>(recvk, nk, d->lo, nb, d->tcount);
+        DCUDA(g, cudaGetLastError());
+        unsigned long long* k1 = nullptr;
+        DCUDA(g, cudaMalloc(&k1, nk * sizeof(unsigned long long)));
+        cub::DoubleBuffer<unsigned long long> db(recvk, k1);
         size_t tb = 0;
-        DCUDA(d, cub::DeviceRadixSort::SortKeys(nullptr, tb, db, nk, 0, nb_row + nb, d->stream));
+        DCUDA(g, cub::DeviceRadixSort::SortKeys(nullptr, tb, db, nk, 0, 64, g->stream));
         void* tmp = nullptr;
-        DCUDA(d, cudaMalloc(&tmp, tb));
-        DCUDA(d, cub::DeviceRadixSort::SortKeys(tmp, tb, db, nk, 0, nb_row + nb, d->stream));
+        DCUDA(g, cudaMalloc(&tmp, tb));
+        DCUDA(g, cub::DeviceRadixSort::SortKeys(tmp, tb, db, nk, 0, 64, g->stream));
         cudaFree(tmp);
         unsigned long long* sorted = db.Current();
         unsigned long long* other = db.Alternate();
         long long* nsel = nullptr;
-        DCUDA(d, cudaMalloc(&nsel, sizeof(long long)));
+        DCUDA(g, cudaMalloc(&nsel, sizeof(long long)));
         size_t ub = 0;
-        DCUDA(d, cub::DeviceSelect::Unique(nullptr, ub, sorted, other, nsel, nk, d->stream));
-        DCUDA(d, cudaMalloc(&tmp, ub));
-        DCUDA(d, cub::DeviceSelect::Unique(tmp, ub, sorted, other, nsel, nk, d->stream));
-        DCUDA(d, cudaMemcpyAsync(&arcs, nsel, sizeof(long long), cudaMemcpyDeviceToHost, d->stream));
-        DCUDA(d, cudaStreamSynchronize(d->stream));
+        DCUDA(g, cub::DeviceSelect::Unique(nullptr, ub, sorted, other, nsel, nk, g->stream));
+        DCUDA(g, cudaMalloc(&tmp, ub));
+        DCUDA(g, cub::DeviceSelect::Unique(tmp, ub, sorted, other, nsel, nk, g->stream));
+        DCUDA(g, cudaMemcpyAsync(&arcs, nsel, sizeof(long long), cudaMemcpyDeviceToHost, g->stream));
+        DCUDA(g, cudaStreamSynchronize(g->stream));
         cudaFree(tmp);
         cudaFree(nsel);
-        DCUDA(d, cudaMalloc(&d->col, std::max(arcs, 1ll) * sizeof(int)));
-        k_split<<<grid_for(arcs), kB, 0, d->stream>>>(other, arcs, count, nb, d->col, d->row_ptr);
-        DCUDA(d, cudaGetLastError());
+        if (arcs > 0) {                          // the self-loop sentinel sorts last
+            unsigned long long last = 0;
+            DCUDA(g, cudaMemcpy(&last, other + arcs - 1, sizeof(last), cudaMemcpyDeviceToHost));
+            if (last == kDrop) --arcs;
+        }
+        DCUDA(g, cudaMalloc(&d->col, std::max(arcs, 1ll) * sizeof(int)));
+        if (arcs > 0) {
+            k_split<<<grid_for(arcs), kB, 0, g->stream>>>(other, arcs, count, nb, d->col, d->row_ptr);
+        } else {
+            k_fill64<<<grid_for(count + 1), kB, 0, g->stream>>>(d->row_ptr, count + 1, 0);
+        }
+        DCUDA(g, cudaGetLastError());
+        DCUDA(g, cudaStreamSynchronize(g->stream));
+        cudaFree(recvk);                         // both key buffers (sorted / other are these two)
+        cudaFree(k1);
+        recvk = nullptr;
     } else {
-        DCUDA(d, cudaMalloc(&d->col, sizeof(int)));
-        k_fill64<<<grid_for(count + 1), kB, 0, d->stream>>>(d->row_ptr, count + 1, 0);
-        DCUDA(d, cudaGetLastError());
+        DCUDA(g, cudaMalloc(&d->col, sizeof(int)));
+        k_fill64<<<grid_for(count + 1), kB, 0, g->stream>>>(d->row_ptr, count + 1, 0);
+        DCUDA(g, cudaGetLastError());
+        if (recvk) cudaFree(recvk);
     }
-    DCUDA(d, cudaStreamSynchronize(d->stream));
-    cudaFree(k0);
-    cudaFree(k1);
-    cudaFree(nkeys);
-    cudaFree(bad);
-    d->arcs = arcs;
-    // degree-aware re-arrangement by global tuple-incidence count (R-6)
+    d->arcs_local = arcs;
+    // 5. true degrees of every vertex (owned slices all-gathered over peer memory),
+    //    then the re-arrangement of every owned row as xbfs_reorder does
+    int* deg_all = nullptr;
+    unsigned* mx = nullptr;
+    DCUDA(g, cudaMalloc(&deg_all, ((long long)nr * d->blk) * sizeof(int)));
+    DCUDA(g, cudaMalloc(&mx, sizeof(unsigned)));
+    DCUDA(g, cudaMemsetAsync(mx, 0, sizeof(unsigned), g->stream));
+    int* my_deg = deg_all + (long long)me * d->blk;
+    if (count > 0) k_degrees<<<grid_for(count), kB, 0, g->stream>>>(d->row_ptr, count, my_deg, mx);
+    DCUDA(g, cudaGetLastError());
+    unsigned hmx = 0;
+    DCUDA(g, cudaMemcpyAsync(&hmx, mx, sizeof(unsigned), cudaMemcpyDeviceToHost, g->stream));
+    DCUDA(g, cudaStreamSynchronize(g->stream));
+    cudaFree(mx);
+    {
+        void* peers[XBFS_DIST_MAX_RANKS];
+        DTRY(exchange_handles(g, c, deg_all, peers));
+        for (int p = 0; p < nr; ++p) {
+            if (p == me || !peers[p]) continue;
+            const long long plo = std::min<long long>(n, (long long)p * d->blk);
+            const long long pc = std::max(0ll, std::min<long long>(d->blk, n - plo));
+            if (pc > 0)
+                DCUDA(g, cudaMemcpyAsync(deg_all + (long long)p * d->blk, (int*)peers[p] + (long long)p * d->blk,
+                                         pc * sizeof(int), cudaMemcpyDefault, g->stream));
+        }
+        DCUDA(g, cudaStreamSynchronize(g->stream));
+        DTRY(comm_barrier(c));
+        close_handles(c, peers);
+    }
+    int64_t gl[4] = {arcs, (int64_t)hmx, 0, 0}, gsum[4];
+    {
+        std::vector<int64_t> allmx(nr * 4);
+        DTRY(comm_allgather(c, gl, sizeof(gl), allmx.data()));
+        gsum[0] = 0;
+        gsum[1] = 0;
+        for (int p = 0; p < nr; ++p) {
+            gsum[0] += allmx[p * 4];
+            gsum[1] = std::max<int64_t>(gsum[1], allmx[p * 4 + 1]);
+        }
+    }
+    d->arcs_global = gsum[0];
+    const unsigned long long maxdeg = (unsigned long long)gsum[1];
+    g->max_deg = (int)maxdeg;
     if (arcs > 0) {
-        unsigned* mx = nullptr;
-        DCUDA(d, cudaMalloc(&mx, sizeof(unsigned)));
-        DCUDA(d, cudaMemsetAsync(mx, 0, sizeof(unsigned), d->stream));
-        k_maxinc<<<grid_for(n), kB, 0, d->stream>>>(inc, n, mx);
-        unsigned hmx = 0;
-        DCUDA(d, cudaMemcpyAsync(&hmx, mx, sizeof(unsigned), cudaMemcpyDeviceToHost, d->stream));
-        DCUDA(d, cudaStreamSynchronize(d->stream));
-        cudaFree(mx);
-        const int db = std::max(1, bitlen(hmx));
+        const int dbits = std::max(1, bitlen(maxdeg));
         unsigned long long *r0 = nullptr, *r1 = nullptr;
         int* c1 = nullptr;
-        DCUDA(d, cudaMalloc(&r0, arcs * sizeof(unsigned long long)));
-        DCUDA(d, cudaMalloc(&r1, arcs * sizeof(unsigned long long)));
-        DCUDA(d, cudaMalloc(&c1, arcs * sizeof(int)));
-        k_rkeys<<<grid_for(arcs), kB, 0, d->stream>>>(d->row_ptr, d->col, inc, count, arcs, db,
-                                                       (unsigned long long)hmx, r0);
-        DCUDA(d, cudaGetLastError());
+        DCUDA(g, cudaMalloc(&r0, arcs * sizeof(unsigned long long)));
+        DCUDA(g, cudaMalloc(&r1, arcs * sizeof(unsigned long long)));
+        DCUDA(g, cudaMalloc(&c1, arcs * sizeof(int)));
+        k_rkeys<<<grid_for(arcs), kB, 0, g->stream>>>(d->row_ptr, d->col, deg_all, count, arcs, dbits, maxdeg, r0);
+        DCUDA(g, cudaGetLastError());
         cub::DoubleBuffer<unsigned long long> dk(r0, r1);
         cub::DoubleBuffer<int> dv(d->col, c1);
         size_t tb = 0;
-        DCUDA(d, cub::DeviceRadixSort::SortPairs(nullptr, tb, dk, dv, arcs, 0, nb_row + db, d->stream));
+        DCUDA(g, cub::DeviceRadixSort::SortPairs(nullptr, tb, dk, dv, arcs, 0, nb_row + dbits, g->stream));
         void* tmp = nullptr;
-        DCUDA(d, cudaMalloc(&tmp, tb));
-        DCUDA(d, cub::DeviceRadixSort::SortPairs(tmp, tb, dk, dv, arcs, 0, nb_row + db, d->stream));
-        DCUDA(d, cudaStreamSynchronize(d->stream));
+        DCUDA(g, cudaMalloc(&tmp, tb));
+        DCUDA(g, cub::DeviceRadixSort::SortPairs(tmp, tb, dk, dv, arcs, 0, nb_row + dbits, g->stream));
+        DCUDA(g, cudaStreamSynchronize(g->stream));
         cudaFree(tmp);
         if (dv.Current() != d->col) { cudaFree(d->col); d->col = dv.Current(); } else { cudaFree(c1); }
         cudaFree(r0);
         cudaFree(r1);
     }
-    cudaFree(inc);
-    // per-vertex facts and BFS state
-    DCUDA(d, cudaMalloc(&d->head, std::max(count, 1ll) * sizeof(unsigned long long)));
-    DCUDA(d, cudaMalloc(&d->noniso, std::max(d->cw, 1ll) * sizeof(unsigned)));
-    DCUDA(d, cudaMalloc(&d->vis, std::max(d->cw, 1ll) * sizeof(unsigned)));
-    DCUDA(d, cudaMalloc(&d->acc, sizeof(DAcc)));
-    DCUDA(d, cudaMemsetAsync(d->acc, 0, sizeof(DAcc), d->stream));
-    DCUDA(d, cudaHostAlloc(&d->acc_host, sizeof(DAcc), cudaHostAllocDefault));
-    k_facts<<<grid_for(d->cw), kB, 0, d->stream>>>(d->row_ptr, d->col, count, d->cw, d->noniso, d->head,
+    DTRY(comm_barrier(c));                  // every peer has copied my degree slice
+    cudaFree(deg_all);
+    // 6. per-vertex facts, BFS state, the shared region every peer maps
+    DCUDA(g, cudaMalloc(&d->head, std::max(count, 1ll) * sizeof(unsigned long long)));
+    DCUDA(g, cudaMalloc(&d->noniso, std::max(d->cw, 1ll) * sizeof(unsigned)));
+    DCUDA(g, cudaMalloc(&d->vis, std::max(d->cw, 1ll) * sizeof(unsigned)));
+    DCUDA(g, cudaMalloc(&d->acc, sizeof(DAcc)));
+    DCUDA(g, cudaMemsetAsync(d->acc, 0, sizeof(DAcc), g->stream));
+    DCUDA(g, cudaHostAlloc(&d->acc_host, sizeof(DAcc), cudaHostAllocDefault));
+    k_facts<<<grid_for(d->cw), kB, 0, g->stream>>>(d->row_ptr, d->col, count, d->cw, d->noniso, d->head,
                                                    &d->acc->found);
-    DCUDA(d, cudaGetLastError());
-    DCUDA(d, cudaMemcpyAsync(d->acc_host, d->acc, sizeof(DAcc), cudaMemcpyDeviceToHost, d->stream));
-    DCUDA(d, cudaStreamSynchronize(d->stream));
+    DCUDA(g, cudaGetLastError());
+    DCUDA(g, cudaMemcpyAsync(d->acc_host, d->acc, sizeof(DAcc), cudaMemcpyDeviceToHost, g->stream));
+    DCUDA(g, cudaStreamSynchronize(g->stream));
     d->nonisolated_local = (long long)d->acc_host->found;
-    DCUDA(d, cudaMemsetAsync(d->acc, 0, sizeof(DAcc), d->stream));
-    // TD work items: one per 1024-arc chunk, at most arcs/1024 + count
+    DCUDA(g, cudaMemsetAsync(d->acc, 0, sizeof(DAcc), g->stream));
+    {
+        int64_t in[2] = {d->nonisolated_local, 0}, out[2];
+        DTRY(comm_allreduce_sum(c, in, out, 2));
+        d->nonisolated_global = out[0];
+    }
     d->items_cap = arcs / kChunkArcs + count + 1;
-    DCUDA(d, cudaMalloc(&d->items, d->items_cap * sizeof(unsigned long long)));
-    // shared region: 3 replicated frontier bitmaps + inbox
+    DCUDA(g, cudaMalloc(&d->items, d->items_cap * sizeof(unsigned long long)));
     const size_t sh = (3 * d->fwords_pad + d->blk_w) * sizeof(unsigned);
-    DCUDA(d, cudaMalloc(&d->shared, sh));
-    DCUDA(d, cudaMemsetAsync(d->shared, 0, sh, d->stream));
-    DCUDA(d, cudaStreamSynchronize(d->stream));
-    return XBFS_OK;
-}
-
-xbfs_status check(xbfs_dist* d) {
-    if (!d) return set_error(XBFS_ERR_INVALID_ARG, "NULL dist handle");
-    if (d->poisoned) return set_error(XBFS_ERR_STATE, "dist handle poisoned by an earlier failure");
+    DCUDA(g, cudaMalloc(&d->shared, sh));
+    DCUDA(g, cudaMemsetAsync(d->shared, 0, sh, g->stream));
+    DCUDA(g, cudaStreamSynchronize(g->stream));
+    {
+        void* peers[XBFS_DIST_MAX_RANKS];
+        DTRY(exchange_handles(g, c, d->shared, peers));
+        for (int p = 0; p < nr; ++p) d->peer_base[p] = p == me ? nullptr : (unsigned*)peers[p];
+    }
+    DCUDA(g, cudaEventCreate(&d->ev0));
+    DCUDA(g, cudaEventCreate(&d->ev1));
+    DTRY(comm_barrier(c));
     return XBFS_OK;
 }
 
@@ -630,227 +798,163 @@ xbfs_status check(xbfs_dist* d) {
 
 extern "C" {
 
-xbfs_status xbfs_dist_build(const void* src, const void* dst, int64_t m, int64_t n, int32_t nranks, int32_t rank,
-                            const xbfs_build_opts* opts, xbfs_dist** out) {
-    if (!out) return set_error(XBFS_ERR_INVALID_ARG, "xbfs_dist_build: out is NULL");
+xbfs_status xbfs_build_csr_dist(xbfs_comm* c, const void* src, const void* dst, int64_t m, int64_t n,
+                                const xbfs_build_opts* opts, xbfs_graph** out) {
+    if (!out) return set_error(XBFS_ERR_INVALID_ARG, "xbfs_build_csr_dist: out is NULL");
     *out = nullptr;
+    if (!c) return set_error(XBFS_ERR_INVALID_ARG, "xbfs_build_csr_dist: NULL comm");
     if (n <= 0 || n >= (1ll << 31)) return set_error(XBFS_ERR_INVALID_ARG, "num_vertices %lld out of (0, 2^31)", (long long)n);
     if (m < 0 || (m > 0 && (!src || !dst))) return set_error(XBFS_ERR_INVALID_ARG, "bad edge arrays");
-    if (nranks < 1 || nranks > XBFS_DIST_MAX_RANKS || rank < 0 || rank >= nranks)
-        return set_error(XBFS_ERR_INVALID_ARG, "rank %d / nranks %d invalid", rank, nranks);
     xbfs_build_opts o{};
     if (opts) o = *opts;
     if (o.id_bytes == 0) o.id_bytes = 4;
     if (o.id_bytes != 4 && o.id_bytes != 8) return set_error(XBFS_ERR_INVALID_ARG, "id_bytes must be 4 or 8");
     if (o.directed) return set_error(XBFS_ERR_UNSUPPORTED, "directed graphs are single-GPU only (xbfs_build_csr)");
-    xbfs_dist* d = new (std::nothrow) xbfs_dist();
-    if (!d) return set_error(XBFS_ERR_OUT_OF_MEMORY, "host allocation failed");
+    xbfs_graph* g = new (std::nothrow) xbfs_graph();
+    xbfs_dist_part* d = new (std::nothrow) xbfs_dist_part();
+    if (!g || !d) { delete g; delete d; return set_error(XBFS_ERR_OUT_OF_MEMORY, "host allocation failed"); }
+    g->dist = d;
+    struct Guard {
+        xbfs_graph*& g;
+        bool keep = false;
+        ~Guard() { if (!keep) xbfs_destroy(g); }
+    } guard{g};
     if (o.device >= 0) {
-        if (cudaSetDevice(o.device) != cudaSuccess) { delete d; return set_error(XBFS_ERR_CUDA, "cudaSetDevice"); }
-        d->device = o.device;
+        XBFS_CUDA(g, cudaSetDevice(o.device));
+        g->device = o.device;
     } else {
-        cudaGetDevice(&d->device);
+        XBFS_CUDA(g, cudaGetDevice(&g->device));
     }
-    d->stream = (cudaStream_t)o.stream;
-    d->rank = rank;
-    d->nranks = nranks;
+    g->stream = (cudaStream_t)o.stream;
+    XBFS_CUDA(g, cudaDeviceGetAttribute(&g->num_sms, cudaDevAttrMultiProcessorCount, g->device));
+    d->comm = c;
+    d->rank = comm_rank(c);
+    d->nranks = comm_size(c);
     d->n = n;
-    d->blk = ((n + 32LL * nranks - 1) / (32LL * nranks)) * 32;
+    d->blk = ((n + 32LL * d->nranks - 1) / (32LL * d->nranks)) * 32;
     d->blk_w = d->blk / 32;
-    d->lo = std::min<long long>(n, (long long)rank * d->blk);
+    d->lo = std::min<long long>(n, (long long)d->rank * d->blk);
     d->count = std::max(0ll, std::min<long long>(d->blk, n - d->lo));
     d->cw = (d->count + 31) / 32;
     d->fwords = (n + 31) / 32;
     d->fwords_pad = (d->fwords + 31) / 32 * 32;
-    xbfs_run_opts_default(&d->opts);
-    xbfs_status s = build_impl(d, src, dst, m, o);
-    if (s != XBFS_OK) { xbfs_dist_destroy(d); return s; }
-    *out = d;
-    return XBFS_OK;
-}
-
-xbfs_status xbfs_dist_info(const xbfs_dist* d, int64_t* first, int64_t* count, int64_t* local_arcs, int64_t* nv) {
-    if (!d) return set_error(XBFS_ERR_INVALID_ARG, "NULL dist handle");
-    if (first) *first = d->lo;
-    if (count) *count = d->count;
-    if (local_arcs) *local_arcs = d->arcs;
-    if (nv) *nv = d->n;
-    return XBFS_OK;
-}
-
-xbfs_status xbfs_dist_export(xbfs_dist* d, void* handle_out) {
-    xbfs_status s = check(d);
-    if (s != XBFS_OK) return s;
-    if (!handle_out) return set_error(XBFS_ERR_INVALID_ARG, "NULL handle_out");
-    static_assert(sizeof(cudaIpcMemHandle_t) == XBFS_IPC_HANDLE_BYTES, "IPC handle size");
-    cudaIpcMemHandle_t h;
-    DCUDA(d, cudaSetDevice(d->device));
-    DCUDA(d, cudaIpcGetMemHandle(&h, d->shared));
-    memcpy(handle_out, &h, sizeof(h));
-    return XBFS_OK;
-}
-
-xbfs_status xbfs_dist_attach(xbfs_dist* d, const void* handles) {
-    xbfs_status s = check(d);
-    if (s != XBFS_OK) return s;
-    if (!handles) return set_error(XBFS_ERR_INVALID_ARG, "NULL handles");
-    if (d->attached) return set_error(XBFS_ERR_STATE, "already attached");
-    DCUDA(d, cudaSetDevice(d->device));
-    for (int p = 0; p < d->nranks; ++p) {
-        if (p == d->rank) continue;
-        cudaIpcMemHandle_t h;
-        memcpy(&h, (const char*)handles + (size_t)p * XBFS_IPC_HANDLE_BYTES, sizeof(h));
-        void* ptr = nullptr;
-        DCUDA(d, cudaIpcOpenMemHandle(&ptr, h, cudaIpcMemLazyEnablePeerAccess));
-        d->peer_base[p] = (unsigned*)ptr;
+    g->n = n;
+    XBFS_TRY_D(build_dist(g, d, src, dst, m, o));
+    {
+        int64_t in[2] = {m, 0}, outv[2];
+        XBFS_TRY_D(comm_allreduce_sum(c, in, outv, 2));
+        g->m_input = outv[0];
     }
-    d->attached = true;
+    g->arcs = d->arcs_global;
+    guard.keep = true;
+    *out = g;
     return XBFS_OK;
 }
 
-xbfs_status xbfs_dist_begin(xbfs_dist* d, int64_t source, int32_t* level, int32_t* parent,
-                            const xbfs_run_opts* opts, int64_t counts[XBFS_DIST_NCOUNTS]) {
-    xbfs_status s = check(d);
-    if (s != XBFS_OK) return s;
-    if (!d->attached && d->nranks > 1) return set_error(XBFS_ERR_STATE, "xbfs_dist_attach first");
+xbfs_status xbfs_partition_range(const xbfs_graph* g, int64_t* first, int64_t* count) {
+    if (!g) return set_error(XBFS_ERR_INVALID_ARG, "xbfs_partition_range: NULL handle");
+    if (!g->dist) {   // a single-GPU handle owns everything
+        if (first) *first = 0;
+        if (count) *count = g->n;
+        return XBFS_OK;
+    }
+    if (first) *first = g->dist->lo;
+    if (count) *count = g->dist->count;
+    return XBFS_OK;
+}
+
+xbfs_status xbfs_run_dist(xbfs_graph* g, int64_t source, int32_t* level, int32_t* parent, const xbfs_run_opts* opts,
+                          xbfs_run_stats* stats) {
+    if (!g) return set_error(XBFS_ERR_INVALID_ARG, "xbfs_run_dist: NULL handle");
+    xbfs_dist_part* d = g->dist;
+    if (!d) return set_error(XBFS_ERR_STATE, "xbfs_run_dist: not a distributed handle (xbfs_build_csr_dist)");
+    if (g->poisoned) return set_error(XBFS_ERR_STATE, "handle poisoned by an earlier failure");
     if ((!level || !parent) && d->count > 0) return set_error(XBFS_ERR_INVALID_ARG, "NULL level/parent");
-    if (source < 0 || source >= d->n) return set_error(XBFS_ERR_INVALID_ARG, "source out of range");
-    if (!counts) return set_error(XBFS_ERR_INVALID_ARG, "NULL counts");
-    xbfs_run_opts_default(&d->opts);
-    if (opts) d->opts = *opts;
-    if (d->opts.force_strategy < -1 || d->opts.force_strategy > 2)
+    if (source < 0 || source >= d->n) return set_error(XBFS_ERR_INVALID_ARG, "source %lld outside [0, %lld)",
+                                                       (long long)source, d->n);
+    xbfs_run_opts o;
+    xbfs_run_opts_default(&o);
+    if (opts) o = *opts;
+    if (o.force_strategy < -1 || o.force_strategy > 2)
         return set_error(XBFS_ERR_INVALID_ARG, "force_strategy must be -1..2");
-    DCUDA(d, cudaSetDevice(d->device));
-    d->level = level;
-    d->parent = parent;
-    DArgs a = d->args();
-    k_init<<<grid_for(std::max(d->fwords, d->count)), kB, 0, d->stream>>>(a);
-    k_seed<<<1, 1, 0, d->stream>>>(a, source);
-    DCUDA(d, cudaGetLastError());
-    long long deg = 0, tc = 0;
-    const bool owner = source >= d->lo && source < d->lo + d->count;
-    if (owner) {
+    XBFS_CUDA(g, cudaSetDevice(g->device));
+    xbfs_comm* c = d->comm;
+    const DArgs a = d->args(level, parent);
+    cudaStream_t s = g->stream;
+    XBFS_CUDA(g, cudaEventRecord(d->ev0, s));
+    k_init<<<grid_for(std::max(d->fwords, d->count)), kB, 0, s>>>(a);
+    k_seed<<<1, 1, 0, s>>>(a, source);
+    XBFS_CUDA(g, cudaGetLastError());
+    // the source's facts from its owner: {owns, deg, tuples}; all ranks' sum
+    int64_t cnt[4] = {0, 0, 0, 0}, gc[4];
+    if (source >= d->lo && source < d->lo + d->count) {
         unsigned long long hd = 0;
         int t = 0;
-        DCUDA(d, cudaMemcpyAsync(&hd, d->head + (source - d->lo), sizeof(hd), cudaMemcpyDeviceToHost, d->stream));
-        DCUDA(d, cudaMemcpyAsync(&t, d->tcount + (source - d->lo), sizeof(t), cudaMemcpyDeviceToHost, d->stream));
-        DCUDA(d, cudaStreamSynchronize(d->stream));
-        deg = (long long)(hd >> 32);
-        tc = t;
+        XBFS_CUDA(g, cudaMemcpyAsync(&hd, d->head + (source - d->lo), sizeof(hd), cudaMemcpyDeviceToHost, s));
+        XBFS_CUDA(g, cudaMemcpyAsync(&t, d->tcount + (source - d->lo), sizeof(t), cudaMemcpyDeviceToHost, s));
+        cnt[0] = 1;
+        cnt[1] = (int64_t)(hd >> 32);
+        cnt[2] = t;
     }
-    DCUDA(d, cudaStreamSynchronize(d->stream));
-    for (int i = 0; i < XBFS_DIST_NCOUNTS; ++i) counts[i] = 0;
-    counts[0] = owner ? 1 : 0;
-    counts[1] = deg;
-    counts[2] = tc;
-    counts[3] = d->nonisolated_local;
-    counts[4] = d->arcs;
-    d->k = 0;
-    d->started = 0;
-    d->log_s.clear();
-    d->log_f.clear();
-    d->log_e.clear();
-    return XBFS_OK;
-}
-
-xbfs_status xbfs_dist_level(xbfs_dist* d, int32_t phase, int64_t counts[XBFS_DIST_NCOUNTS]) {
-    xbfs_status s = check(d);
-    if (s != XBFS_OK) return s;
-    if (!d->started) return set_error(XBFS_ERR_STATE, "xbfs_dist_advance must follow xbfs_dist_begin");
-    if (!counts || (phase != 0 && phase != 1)) return set_error(XBFS_ERR_INVALID_ARG, "bad phase/counts");
-    DCUDA(d, cudaSetDevice(d->device));
-    DArgs a = d->args();
-    const int k = d->k;
+    XBFS_CUDA(g, cudaStreamSynchronize(s));
+    XBFS_TRY_D(comm_allreduce_sum(c, cnt, gc, 4));      // also: every rank has seeded its replica
+    long long fsize = gc[0], fedges = gc[1], m_total = gc[2], fprev = 0;
+    long long unvisited = d->nonisolated_global - (gc[1] > 0 ? 1 : 0);
+    long long reached = 0, arcs_tr = 0;
+    int strategy = choose(o, d->arcs_global, fsize, 0, fedges, unvisited, -1);
+    int k = 0;
     const int grid = grid_for(std::max(d->fwords, d->cw) * 4, 148 * 8);
-    for (int i = 0; i < XBFS_DIST_NCOUNTS; ++i) counts[i] = 0;
-    if (d->strategy == XBFS_BU) {
-        if (phase == 0) {
-            DCUDA(d, cudaMemsetAsync(d->acc, 0, sizeof(DAcc), d->stream));
-            int nsm = 148;
-            cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, d->device);
-            k_bu<<<nsm * 5, kBuThreads, 0, d->stream>>>(a, k);
-            DCUDA(d, cudaGetLastError());
+    const int cap = stats ? stats->level_capacity : 0;
+    while (fsize > 0) {
+        if (stats && k < cap) {
+            if (stats->strategy) stats->strategy[k] = (int8_t)strategy;
+            if (stats->frontier_vertices) stats->frontier_vertices[k] = fsize;
+            if (stats->frontier_edges) stats->frontier_edges[k] = fedges;
+            if (stats->unvisited) stats->unvisited[k] = unvisited;
         }
-    } else if (phase == 0) {
-        DCUDA(d, cudaMemsetAsync(d->acc, 0, sizeof(DAcc), d->stream));
-        k_items<<<grid, kB, 0, d->stream>>>(a, k);
-        k_td<<<grid, kB, 0, d->stream>>>(a, k);
-        DCUDA(d, cudaGetLastError());
-    } else {
-        k_merge<<<grid, kB, 0, d->stream>>>(a, k);
-        DCUDA(d, cudaGetLastError());
+        XBFS_CUDA(g, cudaMemsetAsync(d->acc, 0, sizeof(DAcc), s));
+        if (strategy == XBFS_BU) {
+            k_bu<<<g->num_sms * 5, kBuThreads, 0, s>>>(a, k);
+        } else {
+            k_items<<<grid, kB, 0, s>>>(a, k);
+            k_td<<<grid, kB, 0, s>>>(a, k);
+            XBFS_CUDA(g, cudaGetLastError());
+            XBFS_CUDA(g, cudaStreamSynchronize(s));
+            XBFS_TRY_D(comm_barrier(c));               // every remote discovery is in its owner's inbox
+            k_merge<<<grid, kB, 0, s>>>(a, k);
+        }
+        XBFS_CUDA(g, cudaGetLastError());
+        XBFS_CUDA(g, cudaMemcpyAsync(d->acc_host, d->acc, sizeof(DAcc), cudaMemcpyDeviceToHost, s));
+        XBFS_CUDA(g, cudaStreamSynchronize(s));
+        int64_t lc[4] = {(int64_t)d->acc_host->found, (int64_t)d->acc_host->edges, (int64_t)d->acc_host->m,
+                         (int64_t)d->acc_host->probes};
+        XBFS_TRY_D(comm_allreduce_sum(c, lc, gc, 4));  // also orders this level's peer stores before the next
+        if (stats && k < cap && stats->bu_probes) stats->bu_probes[k] = strategy == XBFS_BU ? gc[3] : 0;
+        reached += fsize;
+        arcs_tr += fedges;
+        fprev = fsize;
+        fsize = gc[0];
+        fedges = gc[1];
+        m_total += gc[2];
+        unvisited -= gc[0];
+        ++k;
+        if (fsize > 0) strategy = choose(o, d->arcs_global, fsize, fprev, fedges, unvisited, strategy);
     }
-    DCUDA(d, cudaMemcpyAsync(d->acc_host, d->acc, sizeof(DAcc), cudaMemcpyDeviceToHost, d->stream));
-    DCUDA(d, cudaStreamSynchronize(d->stream));
-    const bool last = d->strategy == XBFS_BU ? phase == 0 : phase == 1;
-    if (last) {
-        counts[0] = (int64_t)d->acc_host->found;
-        counts[1] = (int64_t)d->acc_host->edges;
-        counts[2] = (int64_t)d->acc_host->m;
-        counts[3] = (int64_t)d->acc_host->probes;
+    XBFS_CUDA(g, cudaEventRecord(d->ev1, s));
+    XBFS_CUDA(g, cudaEventSynchronize(d->ev1));
+    if (stats) {
+        float ms = 0.f;
+        XBFS_CUDA(g, cudaEventElapsedTime(&ms, d->ev0, d->ev1));
+        stats->elapsed_ms = ms;
+        stats->num_levels = k;
+        stats->vertices_reached = reached;
+        stats->arcs_traversed = arcs_tr;
+        stats->input_edges_traversed = m_total;
+        stats->kernel_launches = 0;
+        stats->num_kernels = 0;
+        stats->init_ms = 0.f;
     }
     return XBFS_OK;
-}
-
-xbfs_status xbfs_dist_advance(xbfs_dist* d, const int64_t g[XBFS_DIST_NCOUNTS], int32_t* strategy_out,
-                              int32_t* done) {
-    xbfs_status s = check(d);
-    if (s != XBFS_OK) return s;
-    if (!g) return set_error(XBFS_ERR_INVALID_ARG, "NULL counts");
-    if (!d->started) {
-        // first call: g = {1, deg(s), tcount(s), non-isolated vertices, arcs A}
-        d->fsize = g[0];
-        d->fedges = g[1];
-        d->m_total = g[2];
-        d->unvisited = g[3] - (g[1] > 0 ? 1 : 0);
-        d->arcs_global = g[4];
-        d->fprev = 0;
-        d->started = 1;
-        d->strategy = choose(d->opts, d->arcs_global, d->fsize, 0, d->fedges, d->unvisited, -1);
-    } else {
-        d->log_s.push_back((int8_t)d->strategy);
-        d->log_f.push_back(d->fsize);
-        d->log_e.push_back(d->fedges);
-        const int prev = d->strategy;
-        d->fprev = d->fsize;
-        d->fsize = g[0];
-        d->fedges = g[1];
-        d->m_total += g[2];
-        d->unvisited -= g[0];
-        d->k += 1;
-        d->strategy = choose(d->opts, d->arcs_global, d->fsize, d->fprev, d->fedges, d->unvisited, prev);
-    }
-    if (strategy_out) *strategy_out = d->strategy;
-    if (done) *done = d->fsize == 0 ? 1 : 0;
-    return XBFS_OK;
-}
-
-xbfs_status xbfs_dist_levels(const xbfs_dist* d, int32_t cap, int8_t* strategy, int64_t* fv, int64_t* fe,
-                             int32_t* num_levels, int64_t* input_edges) {
-    if (!d) return set_error(XBFS_ERR_INVALID_ARG, "NULL dist handle");
-    const int nl = (int)d->log_s.size();
-    for (int i = 0; i < std::min(nl, cap); ++i) {
-        if (strategy) strategy[i] = d->log_s[i];
-        if (fv) fv[i] = d->log_f[i];
-        if (fe) fe[i] = d->log_e[i];
-    }
-    if (num_levels) *num_levels = nl;
-    if (input_edges) *input_edges = d->m_total;
-    return XBFS_OK;
-}
-
-void xbfs_dist_destroy(xbfs_dist* d) {
-    if (!d) return;
-    cudaSetDevice(d->device);
-    if (d->stream) cudaStreamSynchronize(d->stream);
-    for (int p = 0; p < XBFS_DIST_MAX_RANKS; ++p)
-        if (d->peer_base[p]) cudaIpcCloseMemHandle(d->peer_base[p]);
-    void* ptrs[] = {d->row_ptr, d->col, d->head, d->tcount, d->noniso, d->vis, d->shared, d->items, d->acc};
-    for (void* p : ptrs)
-        if (p) cudaFree(p);
-    if (d->acc_host) cudaFreeHost(d->acc_host);
-    cudaGetLastError();
-    delete d;
 }
 
 }  // extern "C"

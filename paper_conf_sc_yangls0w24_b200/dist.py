@@ -1,125 +1,111 @@
-"""Multi-GPU XBFS driver (include/xbfs_dist.h): 1D vertex partition, one process
-per GPU, torch.distributed for the plumbing (IPC-handle exchange, the 8-counter
-all-reduce and the barrier between the two phases of a top-down level).
-
-All per-level compute and the frontier exchange run in libxbfs.so: bottom-up
-levels publish their owned next-frontier words straight into every peer's
-replica, top-down levels OR remote discoveries into the owner's inbox in peer
-memory (north_star "direction switch made on globally reduced
-counts").  This module only sequences the calls.
+"""Multi-GPU XBFS binding (include/xbfs_dist.h): 1D vertex partition, one
+process per GPU.  Argument marshalling only: the communicator (a shared-memory
+segment on the node, reading R-10), the distributed CSR build with its
+peer-memory arc shuffle, and every level of xbfs_run_dist (kernels, peer-memory
+frontier exchange, barriers, the per-level counter all-reduce) run inside
+libxbfs.so.  torch.distributed is used once, to broadcast the 128-byte unique id
+from rank 0 (as one would an ncclUniqueId).
 """
 from __future__ import annotations
 
 import ctypes
-from dataclasses import dataclass, field
 
 import numpy as np
 
 from . import xbfs as _x
 
-NCOUNTS = 8
-IPC_BYTES = 64
-BU = _x.BU
+UNIQUE_ID_BYTES = 128
+MAX_RANKS = 16
 
 _L = _x.lib
 _P, _i64, _i32 = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int32
-_L.xbfs_dist_build.argtypes = [_P, _P, _i64, _i64, _i32, _i32, ctypes.POINTER(_x.BuildOpts), ctypes.POINTER(_P)]
-_L.xbfs_dist_info.argtypes = [_P, _P, _P, _P, _P]
-_L.xbfs_dist_export.argtypes = [_P, _P]
-_L.xbfs_dist_attach.argtypes = [_P, _P]
-_L.xbfs_dist_begin.argtypes = [_P, _i64, _P, _P, ctypes.POINTER(_x.RunOpts), _P]
-_L.xbfs_dist_level.argtypes = [_P, _i32, _P]
-_L.xbfs_dist_advance.argtypes = [_P, _P, _P, _P]
-_L.xbfs_dist_levels.argtypes = [_P, _i32, _P, _P, _P, _P, _P]
-_L.xbfs_dist_destroy.argtypes = [_P]
-_L.xbfs_dist_destroy.restype = None
-for _fn in ("xbfs_dist_build", "xbfs_dist_info", "xbfs_dist_export", "xbfs_dist_attach", "xbfs_dist_begin",
-            "xbfs_dist_level", "xbfs_dist_advance", "xbfs_dist_levels"):
+_L.xbfs_get_unique_id.argtypes = [_P]
+_L.xbfs_comm_init.argtypes = [_P, _i32, _i32, ctypes.POINTER(_P)]
+_L.xbfs_comm_barrier.argtypes = [_P]
+_L.xbfs_comm_allreduce_i64.argtypes = [_P, _P, _P, _i32]
+_L.xbfs_comm_destroy.argtypes = [_P]
+_L.xbfs_comm_destroy.restype = None
+_L.xbfs_build_csr_dist.argtypes = [_P, _P, _P, _i64, _i64, ctypes.POINTER(_x.BuildOpts), ctypes.POINTER(_P)]
+_L.xbfs_partition_range.argtypes = [_P, _P, _P]
+_L.xbfs_run_dist.argtypes = [_P, _i64, _P, _P, ctypes.POINTER(_x.RunOpts), ctypes.POINTER(_x.RunStats)]
+for _fn in ("xbfs_get_unique_id", "xbfs_comm_init", "xbfs_comm_barrier", "xbfs_comm_allreduce_i64",
+            "xbfs_build_csr_dist", "xbfs_partition_range", "xbfs_run_dist"):
     getattr(_L, _fn).restype = ctypes.c_int
 
 #: symbols include/xbfs_dist.h declares (checked by tests/test_abi.py)
-DIST_EXPORTS = ("xbfs_dist_build", "xbfs_dist_info", "xbfs_dist_export", "xbfs_dist_attach", "xbfs_dist_begin",
-                "xbfs_dist_level", "xbfs_dist_advance", "xbfs_dist_levels", "xbfs_dist_destroy")
+DIST_EXPORTS = ("xbfs_get_unique_id", "xbfs_comm_init", "xbfs_comm_barrier", "xbfs_comm_allreduce_i64",
+                "xbfs_build_csr_dist", "xbfs_partition_range", "xbfs_run_dist", "xbfs_comm_destroy")
 
 
 def partition(n: int, nranks: int, rank: int):
-    """Owned range of `rank` (mirrors xbfs_dist_build): blocks of B = 32*ceil(n/(32p))."""
+    """Owned range of `rank` (the library's rule): blocks of B = 32*ceil(n/(32p))."""
     blk = 32 * ((n + 32 * nranks - 1) // (32 * nranks))
     lo = min(n, rank * blk)
     return lo, max(0, min(blk, n - lo))
 
 
-@dataclass
-class DistStats:
-    num_levels: int
-    input_edges_traversed: int
-    strategy: list = field(default_factory=list)
-    frontier_vertices: list = field(default_factory=list)
-    frontier_edges: list = field(default_factory=list)
-    elapsed_ms: float = 0.0
+def tuple_range(m: int, nranks: int, rank: int):
+    """The share of the M input tuples rank `rank` generates / passes to the build."""
+    return rank * m // nranks, (rank + 1) * m // nranks
 
 
-class _LibBackend:
-    """The real per-rank backend: libxbfs.so's xbfs_dist_* entry points."""
-
-    def __init__(self, h):
-        self.h = h
-
-    def begin(self, source, level, parent, opts):
-        c = np.zeros(NCOUNTS, np.int64)
-        _x._check(_L.xbfs_dist_begin(self.h, int(source), _x._ptr(level) if level.numel() else None,
-                                     _x._ptr(parent) if parent.numel() else None, ctypes.byref(opts), c.ctypes.data))
-        return c
-
-    def level(self, phase):
-        c = np.zeros(NCOUNTS, np.int64)
-        _x._check(_L.xbfs_dist_level(self.h, phase, c.ctypes.data))
-        return c
-
-    def advance(self, g):
-        g = np.ascontiguousarray(g, dtype=np.int64)
-        s, d = ctypes.c_int32(), ctypes.c_int32()
-        _x._check(_L.xbfs_dist_advance(self.h, g.ctypes.data, ctypes.byref(s), ctypes.byref(d)))
-        return s.value, bool(d.value)
-
-    def levels(self):
-        cap = 1 << 14
-        st = np.zeros(cap, np.int8)
-        fv = np.zeros(cap, np.int64)
-        fe = np.zeros(cap, np.int64)
-        nl, m = ctypes.c_int32(), ctypes.c_int64()
-        _x._check(_L.xbfs_dist_levels(self.h, cap, st.ctypes.data, fv.ctypes.data, fe.ctypes.data,
-                                      ctypes.byref(nl), ctypes.byref(m)))
-        k = min(nl.value, cap)
-        return DistStats(nl.value, m.value, st[:k].tolist(), fv[:k].tolist(), fe[:k].tolist())
+def xbfs_get_unique_id() -> bytes:
+    buf = (ctypes.c_ubyte * UNIQUE_ID_BYTES)()
+    _x._check(_L.xbfs_get_unique_id(buf))
+    return bytes(buf)
 
 
-def drive(backend, allreduce, barrier, source, level, parent, opts):
-    """The level loop shared by every rank (host-side logic, testable with any
-    backend): begin -> all-reduce -> advance, then per level phase 0, and for a
-    top-down level a barrier and phase 1, then all-reduce -> advance."""
-    g = allreduce(backend.begin(source, level, parent, opts))
-    strategy, done = backend.advance(g)
-    while not done:
-        c = backend.level(0)
-        if strategy != BU:
-            barrier()               # every remote discovery is in its owner's inbox
-            c = backend.level(1)
-        g = allreduce(c)            # also orders this level's peer stores before the next level
-        strategy, done = backend.advance(g)
-    return backend.levels()
+class Comm:
+    """One rank of the node-local communicator.  `uid` must be the same bytes on
+    every rank (rank 0's xbfs_get_unique_id)."""
+
+    def __init__(self, uid: bytes, nranks: int, rank: int):
+        buf = (ctypes.c_ubyte * UNIQUE_ID_BYTES).from_buffer_copy(uid)
+        h = ctypes.c_void_p()
+        _x._check(_L.xbfs_comm_init(buf, int(nranks), int(rank), ctypes.byref(h)))
+        self._h, self.nranks, self.rank = h.value, int(nranks), int(rank)
+
+    @classmethod
+    def from_torch(cls, group=None):
+        """Collective over a torch.distributed group: rank 0 makes the id, broadcast it."""
+        import torch.distributed as dist
+        rank, world = dist.get_rank(group), dist.get_world_size(group)
+        obj = [xbfs_get_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(obj, src=0, group=group)
+        return cls(obj[0], world, rank)
+
+    def barrier(self):
+        _x._check(_L.xbfs_comm_barrier(self._h))
+
+    def allreduce(self, values):
+        a = np.ascontiguousarray(np.asarray(values, dtype=np.int64))
+        out = np.empty_like(a)
+        _x._check(_L.xbfs_comm_allreduce_i64(self._h, a.ctypes.data, out.ctypes.data, int(a.size)))
+        return out
+
+    @property
+    def handle(self):
+        return self._h
+
+    def close(self):
+        if getattr(self, "_h", None):
+            _L.xbfs_comm_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
 
 
 class DistGraph:
-    """One rank's partition of a graph.  Collective: every rank of `group`
-    constructs it with the same full tuple list."""
+    """This rank's partition of a graph (collective over `comm`).  src/dst: THIS
+    rank's share of the input tuples (numpy, or torch tensors on host or device)."""
 
-    def __init__(self, src, dst, num_vertices: int, group=None, device: int | None = None, stream=None):
+    def __init__(self, comm: Comm, src, dst, num_vertices: int, device: int | None = None, stream=None):
         import torch
-        import torch.distributed as dist
-        self.group = group
-        self.rank = dist.get_rank(group)
-        self.world = dist.get_world_size(group)
+        self.comm = comm
         self.device = torch.cuda.current_device() if device is None else device
         if stream is None:
             stream = torch.cuda.current_stream(self.device).cuda_stream
@@ -133,51 +119,33 @@ class DistGraph:
                          keep_duplicates=0)
         m = int(src.shape[0])
         h = ctypes.c_void_p()
-        _x._check(_L.xbfs_dist_build(_x._ptr(src) if m else None, _x._ptr(dst) if m else None, m, num_vertices,
-                                     self.world, self.rank, ctypes.byref(o), ctypes.byref(h)))
+        _x._check(_L.xbfs_build_csr_dist(comm.handle, _x._ptr(src) if m else None, _x._ptr(dst) if m else None, m,
+                                         int(num_vertices), ctypes.byref(o), ctypes.byref(h)))
         self._h = h.value
-        first, count, arcs, n = ctypes.c_int64(), ctypes.c_int64(), ctypes.c_int64(), ctypes.c_int64()
-        _x._check(_L.xbfs_dist_info(self._h, ctypes.byref(first), ctypes.byref(count), ctypes.byref(arcs),
-                                    ctypes.byref(n)))
-        self.first, self.count, self.local_arcs, self.n = first.value, count.value, arcs.value, n.value
-        buf = (ctypes.c_ubyte * IPC_BYTES)()
-        _x._check(_L.xbfs_dist_export(self._h, buf))
-        handles = [None] * self.world
-        dist.all_gather_object(handles, bytes(buf), group=group)
-        allh = b"".join(handles)
-        _x._check(_L.xbfs_dist_attach(self._h, allh))
-        dist.barrier(group=group)
-        self._backend = _LibBackend(self._h)
-        self._nccl = dist.get_backend(group) == "nccl"
+        first, count = ctypes.c_int64(), ctypes.c_int64()
+        _x._check(_L.xbfs_partition_range(self._h, ctypes.byref(first), ctypes.byref(count)))
+        self.first, self.count = first.value, count.value
+        self.n, self.arcs, self.m_input, self.max_degree = _x.xbfs_graph_info(self._h)
 
-    def _allreduce(self, c):
-        import torch
-        import torch.distributed as dist
-        t = torch.as_tensor(np.asarray(c, dtype=np.int64))
-        if self._nccl:
-            t = t.cuda(self.device)
-        dist.all_reduce(t, group=self.group)
-        return t.cpu().numpy()
-
-    def _barrier(self):
-        import torch.distributed as dist
-        dist.barrier(group=self.group)
-
-    def run(self, source: int, level=None, parent=None, **opts):
-        """BFS from global `source`.  Returns (level_local, parent_local, DistStats)
-        for this rank's owned range [first, first+count)."""
+    def run(self, source: int, level=None, parent=None, stats: bool = True, **opts):
+        """BFS from global `source` (xbfs_run_dist).  Returns (level_local,
+        parent_local, Stats) for this rank's owned range [first, first+count);
+        Stats.elapsed_ms is this rank's device time (take the max over ranks)."""
         import torch
         dev = f"cuda:{self.device}"
         if level is None:
-            level = torch.empty(self.count, dtype=torch.int32, device=dev)
+            level = torch.empty(max(self.count, 1), dtype=torch.int32, device=dev)[: self.count]
         if parent is None:
-            parent = torch.empty(self.count, dtype=torch.int32, device=dev)
-        st = drive(self._backend, self._allreduce, self._barrier, source, level, parent, _x.make_run_opts(**opts))
-        return level, parent, st
+            parent = torch.empty(max(self.count, 1), dtype=torch.int32, device=dev)[: self.count]
+        sb = _x._StatsBuf() if stats else None
+        _x._check(_L.xbfs_run_dist(self._h, int(source), _x._ptr(level) if self.count else None,
+                                   _x._ptr(parent) if self.count else None, ctypes.byref(_x.make_run_opts(**opts)),
+                                   ctypes.byref(sb.c) if sb else None))
+        return level, parent, (sb.result() if sb else None)
 
     def close(self):
         if getattr(self, "_h", None):
-            _L.xbfs_dist_destroy(self._h)
+            _x.xbfs_destroy(self._h)
             self._h = None
 
     def __del__(self):

@@ -21,7 +21,7 @@ def xb():
 def _declared(header):
     txt = open(os.path.join(ROOT, "include", header)).read()
     txt = re.sub(r"/\*.*?\*/", "", txt, flags=re.S)
-    return set(re.findall(r"\b(xbfs_[a-z_]+)\s*\(", txt))
+    return set(re.findall(r"\b(xbfs_[a-z0-9_]+)\s*\(", txt))
 
 
 def test_exports_every_declared_symbol(xb):
@@ -56,10 +56,21 @@ def test_invalid_arguments_do_not_touch_cuda(xb):
     assert xb.lib.xbfs_graph_info(None, None, None, None, None) == xb.XBFS_ERR_INVALID_ARG
     xb.lib.xbfs_destroy(None)  # NULL-safe
     from paper_conf_sc_yangls0w24_b200 import dist
-    assert xb.lib.xbfs_dist_build(None, None, 0, 10, 2, 5, None, ctypes.byref(h)) == xb.XBFS_ERR_INVALID_ARG
-    assert xb.lib.xbfs_dist_build(None, None, 0, 10, 0, 0, None, ctypes.byref(h)) == xb.XBFS_ERR_INVALID_ARG
-    assert xb.lib.xbfs_dist_level(None, 0, None) == xb.XBFS_ERR_INVALID_ARG
-    xb.lib.xbfs_dist_destroy(None)
+    uid = (ctypes.c_ubyte * dist.UNIQUE_ID_BYTES).from_buffer_copy(dist.xbfs_get_unique_id())
+    assert xb.lib.xbfs_comm_init(uid, 2, 5, ctypes.byref(h)) == xb.XBFS_ERR_INVALID_ARG
+    assert xb.lib.xbfs_comm_init(uid, 0, 0, ctypes.byref(h)) == xb.XBFS_ERR_INVALID_ARG
+    assert xb.lib.xbfs_comm_init(uid, 17, 0, ctypes.byref(h)) == xb.XBFS_ERR_INVALID_ARG
+    junk = (ctypes.c_ubyte * dist.UNIQUE_ID_BYTES)()
+    assert xb.lib.xbfs_comm_init(junk, 1, 0, ctypes.byref(h)) == xb.XBFS_ERR_INVALID_ARG
+    assert xb.lib.xbfs_build_csr_dist(None, None, None, 0, 10, None, ctypes.byref(h)) == xb.XBFS_ERR_INVALID_ARG
+    assert xb.lib.xbfs_run_dist(None, 0, None, None, None, None) == xb.XBFS_ERR_INVALID_ARG
+    assert xb.lib.xbfs_partition_range(None, None, None) == xb.XBFS_ERR_INVALID_ARG
+    xb.lib.xbfs_comm_destroy(None)
+    # a one-rank communicator needs no peers and no GPU
+    c = dist.Comm(dist.xbfs_get_unique_id(), 1, 0)
+    assert c.allreduce([1, 2, 3]).tolist() == [1, 2, 3]
+    c.barrier()
+    c.close()
 
 
 def test_product_path_never_imports_oracle():

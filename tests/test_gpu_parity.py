@@ -427,3 +427,87 @@ def test_bench_workload_full_size(xb, cfg):
         st = _check_run(g, og, src, dst, root)
         assert st.kernel_launches == 1          # one cooperative launch per BFS
     g.close()
+
+
+@pytest.mark.parametrize("scale", [16, 20])
+def test_selector_decisions_match_the_rule(xb, scale):
+    """The device selector (every CTA of the persistent kernel steps a replica of it)
+    against oracle_select_sequence: the paper's rule (strict '>' C-8) with
+    the growth rule C-10 and the stay-in-BU hysteresis C-11, replayed on the
+    oracle's exact per-level counters.  The strategy of every level and U_k (the
+    BU candidates before step k) must be identical, for the default options and
+    for other (alpha, grow, ratio_min, bu_stay) settings."""
+    src, dst, n = synth.kronecker(scale, seed=1)
+    og = oracle.build_csr(n, src, dst)
+    g = xb.Graph(_dev(src), _dev(dst), n)
+    d = xb.xbfs_run_opts_default()
+    settings = [dict(alpha=d.alpha, grow=d.grow, ratio_min=d.ratio_min, bu_stay=d.bu_stay),
+                dict(alpha=0.1, grow=2.0, ratio_min=1e-3, bu_stay=0.0),      # the paper's rule
+                dict(alpha=0.01, grow=1.5, ratio_min=1e-4, bu_stay=4.0)]
+    for root in synth.roots(n, src, dst, 6, root_seed=17):
+        ref, _, nl = oracle.bfs(og, int(root))
+        for opt in settings:
+            for drv in (3, 1):
+                _, _, st = g.run(int(root), stats=True, driver=drv, small_edges=0, **opt)
+                want, unv = oracle.select_sequence(og, ref, **opt)
+                assert st.num_levels == nl
+                assert st.strategy == want.tolist(), (root, opt, drv)
+                assert st.unvisited == unv.tolist(), (root, opt, drv)
+    g.close()
+
+
+def test_run_host_batch_pinned_overlap(xb):
+    """xbfs_run_host_batch into PINNED host buffers (the copy of root i really
+    overlaps the BFS of root i+1, so the two device slots' reuse ordering is
+    exercised): 7 roots, every slot's levels exact and parents valid."""
+    src, dst, n = synth.kronecker(14, seed=12)
+    og = oracle.build_csr(n, src, dst)
+    g = xb.Graph(_dev(src), _dev(dst), n)
+    roots = [int(r) for r in synth.roots(n, src, dst, 7, root_seed=21)]
+    k = len(roots)
+    lh = torch.full((k * n,), -7, dtype=torch.int32, pin_memory=True).numpy()
+    ph = torch.full((k * n,), -7, dtype=torch.int32, pin_memory=True).numpy()
+    for _ in range(2):
+        g.run_host_batch(roots, lh, ph)
+        for i, r in enumerate(roots):
+            ref, _, _ = oracle.bfs(og, r)
+            lv, pa = lh[i * n:(i + 1) * n], ph[i * n:(i + 1) * n]
+            assert np.array_equal(lv, ref), i
+            assert oracle.validate(og, src, dst, r, lv, pa) == 0, i
+        lh[:] = -7
+        ph[:] = -7
+    with pytest.raises(ValueError):
+        g.run_host_batch(roots, lh[: n], ph[: n])          # too small for k slots: refused in the binding
+    g.close()
+
+
+def test_bench_workload_s27_full_size(xb):
+    """BASELINE config 4's graph (Kronecker s27 ef16 seed 1: 134 M vertices, 2.1 G
+    tuples, 4.2 G arcs) on one B200 in bench's launch configuration.  Every root
+    checked passes the OpenMP tuple-list Graph500 validator (V1-V5 over all 2.1 G
+    input tuples, which certifies the levels exactly: SURVEY §8(c) O-5), and the
+    first root's levels equal the oracle's serial BFS over its own CSR bit-exactly."""
+    import gc
+
+    import bench
+    src, dst, n = bench.make_graph("s27", pinned=False)
+    roots = [int(r) for r in bench.pick_roots("s27", n, src, dst, 3)]
+    g = xb.Graph(torch.from_numpy(src.view(np.int32)), torch.from_numpy(dst.view(np.int32)), n)
+    results = []
+    for root in roots:
+        level, parent, st = g.run(root, stats=True)
+        assert st.kernel_launches == 1
+        lv, pa = level.cpu().numpy(), parent.cpu().numpy()
+        del level, parent
+        assert oracle.validate_tuples(n, src, dst, root, lv, pa) == 0, root
+        assert st.vertices_reached == int((lv >= 0).sum())
+        results.append((root, lv if not results else None, st))
+    g.close()
+    torch.cuda.empty_cache()
+    gc.collect()
+    root, lv0, st0 = results[0]
+    og = oracle.build_csr(n, src, dst)
+    ref, _, nl = oracle.bfs(og, root)
+    assert np.array_equal(lv0, ref)
+    assert st0.num_levels == nl
+    assert st0.input_edges_traversed == oracle.input_edges(src, ref)
