@@ -291,7 +291,7 @@ __device__ __forceinline__ void seed_body(const KArgs& a, int* level, int* paren
     st->fprev = 0;
     st->unvisited = nonisolated_count - (s_cand ? 1 : 0);
     for (int i = 0; i < 3; ++i) {
-        st->acc_found[i] = st->acc_edges[i] = st->acc_probes[i] = st->acc_zero[i] = 0;
+        st->acc_found[i] = st->acc_edges[i] = st->acc_probes[i] = st->acc_zero[i] = st->bu_gctr[i] = 0;
         st->acc_la_found[i] = st->acc_la_edges[i] = 0;
     }
     st->reached = 0;
@@ -442,6 +442,7 @@ __device__ void select_body(const KArgs& a) {
     st->qmax[(k + 2) % 3] = 0;
     st->acc_found[(k + 1) % 3] = st->acc_edges[(k + 1) % 3] = st->acc_probes[(k + 1) % 3] = 0;
     st->acc_zero[(k + 1) % 3] = 0;
+    st->bu_gctr[(k + 1) % 3] = 0;
     st->acc_la_found[(k + 1) % 3] = st->acc_la_edges[(k + 1) % 3] = 0;
     sel_store(st, s);
     mirror_host(a, st);
@@ -469,6 +470,10 @@ using TdSmem = TdSmemT<1>;
 #endif
 #ifndef XBFS_SF_TPT
 #define XBFS_SF_TPT 1
+#endif
+
+#ifndef XBFS_SS_CLAIM
+#define XBFS_SS_CLAIM 0
 #endif
 
 #ifndef XBFS_SF_PRECHECK_MIN
@@ -587,6 +592,24 @@ __device__ __forceinline__ void td_expand_body(const KArgs& a, int k, int* __res
             // clear write the same level value (benign race; either parent is
             // valid, C-26).  Both bitmaps get fire-and-forget REDs, so later arcs
             // of this level mostly see the vertex as visited (one probe per arc).
+#if XBFS_SS_CLAIM
+            // (variant) the visited RED returns the old word: only the first writer stores
+            unsigned old[R];
+#pragma unroll
+            for (int i = 0; i < R; ++i) {
+                const unsigned bit = 1u << (v[i] & 31);
+                old[i] = (valid[i] && !(vis[i] & bit)) ? atomicOr(visited + (v[i] >> 5), bit) : FULL;
+            }
+#pragma unroll
+            for (int i = 0; i < R; ++i) {
+                const unsigned bit = 1u << (v[i] & 31);
+                if (!(old[i] & bit)) {
+                    level[v[i]] = lvl;
+                    parent[v[i]] = u[i];
+                    atomicOr(next + (v[i] >> 5), bit);
+                }
+            }
+#else
 #pragma unroll
             for (int i = 0; i < R; ++i) {
                 const unsigned bit = 1u << (v[i] & 31);
@@ -597,6 +620,7 @@ __device__ __forceinline__ void td_expand_body(const KArgs& a, int k, int* __res
                     atomicOr(visited + (v[i] >> 5), bit);
                 }
             }
+#endif
         }
     }
     if (MODE == XBFS_SF && a.track_max) flush_max(&a.st->qmax[(k + 1) % 3], lmax);
@@ -739,9 +763,19 @@ __global__ __launch_bounds__(kGenThreads) void k_generate(KArgs a, int role) {
 // kp: where k lives (DevState or the persistent CTA's selector copy); it is
 // re-read for the epilogue instead of keeping k live across the traversal
 // (one register less: the per-level kernel runs at 48 without spills).
+#if XBFS_BU_PROF
+__device__ unsigned long long g_bu_prof[8];   // profiling build: BU phase cycles of the dense steps
+#endif
+
+// Dynamic group scheduling (bu_core.cuh) for dense steps: at least N/16 candidates.
+// (B200 A/B, s24 2x32 roots: dynamic 752 vs static 788 GTEPS: off by default)
+#ifndef XBFS_BU_DYN
+#define XBFS_BU_DYN 0
+#endif
+
 template <int WARPS, bool LA, class Smem, bool DIR = false>
 __device__ __forceinline__ void bu_body(const KArgs& a, const int* kp, int* __restrict__ level,
-                                        int* __restrict__ parent, Smem& sm, bool prefill) {
+                                        int* __restrict__ parent, Smem& sm, bool prefill, long long U) {
     int k = *(const volatile int*)kp;
     clear_stale(a, k);
     const unsigned int* __restrict__ cur = a.fb[k % 3];
@@ -763,6 +797,11 @@ __device__ __forceinline__ void bu_body(const KArgs& a, const int* kp, int* __re
     b.level = level;
     b.parent = parent;
     b.lvl = lvl;
+    b.gctr = (XBFS_BU_DYN && U * 16 >= a.n) ? &a.st->bu_gctr[k % 3] : nullptr;
+    b.dense = U * 16 >= a.n;
+#if XBFS_BU_PROF
+    b.prof = U * 16 >= a.n ? g_bu_prof : nullptr;   // the dense steps only
+#endif
     // prefill: F_{k+1} already holds look-ahead vertices of step k-1 (OR into it)
     const bool pf = LA && prefill;
     unsigned long long oedges = 0;   // DIR: out-degrees of the found vertices, summed where they are published
@@ -839,7 +878,7 @@ __device__ __forceinline__ void la_merge(const KArgs& a, int knext) {
 __global__ __launch_bounds__(kBuThreads, 4) void k_bu_traverse(KArgs a) {
     count_launch(a.st);
     __shared__ BuSmem<kBuThreads / 32> sm;
-    bu_body<kBuThreads / 32, false>(a, &a.st->k, a.st->out_level, a.st->out_parent, sm, false);
+    bu_body<kBuThreads / 32, false>(a, &a.st->k, a.st->out_level, a.st->out_parent, sm, false, a.st->unvisited);
 }
 
 // ---------------------------------------------------------------- select
@@ -1138,16 +1177,17 @@ union PersistSmem {
 // LA: the BU look-ahead variant (a separate instantiation, so the default kernel
 // carries none of its registers).
 // DIR: directed graph (f4, reading R-9; also a separate instantiation).
+// (level / parent are kernel parameters here, not loads from the state: parameters
+// live in the constant bank, registers would be held across the whole kernel)
 template <bool LA, bool DIR>
 __global__ __launch_bounds__(kPersistThreads, kPersistBlocks) void k_persist(
-    KArgs a, const unsigned int* __restrict__ nonisolated, long long nonisolated_count) {
+    KArgs a, int* __restrict__ level, int* __restrict__ parent, const unsigned int* __restrict__ nonisolated,
+    long long nonisolated_count) {
     extern __shared__ __align__(16) unsigned char dsm[];
     PersistSmem<LA>& sm = *reinterpret_cast<PersistSmem<LA>*>(dsm);
     __shared__ SelState s;
     unsigned epoch = 0;
     unsigned* bar = &a.st->bar_count;
-    int* __restrict__ level = a.st->out_level;
-    int* __restrict__ parent = a.st->out_parent;
     if (threadIdx.x == 0) atomicMin(&a.st->t_enter, globaltimer());
     count_launch(a.st);
     // the source's entries are written by the fill itself and the seed state by one
@@ -1167,6 +1207,7 @@ __global__ __launch_bounds__(kPersistThreads, kPersistBlocks) void k_persist(
             a.st->qmax[(k + 2) % 3] = 0;
             a.st->acc_found[(k + 1) % 3] = a.st->acc_edges[(k + 1) % 3] = a.st->acc_probes[(k + 1) % 3] = 0;
             a.st->acc_zero[(k + 1) % 3] = 0;
+            a.st->bu_gctr[(k + 1) % 3] = 0;
             a.st->acc_la_found[(k + 1) % 3] = a.st->acc_la_edges[(k + 1) % 3] = 0;
         }
         if (strat != XBFS_BU && !qvalid) {
@@ -1186,7 +1227,8 @@ __global__ __launch_bounds__(kPersistThreads, kPersistBlocks) void k_persist(
             ss_count_body(a, k);
         } else {
             // (directed: bu_body sums edgesF_{k+1} over out-arcs itself)
-            bu_body<kPersistThreads / 32, LA, decltype(sm.bu), DIR>(a, &s.k, level, parent, sm.bu, s.prefill);
+            bu_body<kPersistThreads / 32, LA, decltype(sm.bu), DIR>(a, &s.k, level, parent, sm.bu, s.prefill,
+                                                                   s.unvisited);
         }
         grid_sync(bar, epoch);
         if (threadIdx.x == 0) select_step(a, s, blockIdx.x == 0, blockIdx.x == 0 ? globaltimer() : 0ull);
@@ -1431,7 +1473,7 @@ xbfs_status build_loop_graph(xbfs_graph* g) {
     return XBFS_OK;
 }
 
-xbfs_status launch_persist(xbfs_graph* g, const KArgs& a, bool lookahead) {
+xbfs_status launch_persist(xbfs_graph* g, const KArgs& a, int* level, int* parent, bool lookahead) {
     static int occ[3][64];
     static bool init[3][64] = {{false}};
     const int dev = g->device & 63, v = lookahead ? 1 : (g->directed ? 2 : 0);
@@ -1451,7 +1493,7 @@ xbfs_status launch_persist(xbfs_graph* g, const KArgs& a, bool lookahead) {
     long long nic = g->nonisolated_count;
     KArgs ka = a;
     ka.track_max = 0;   // no small-frontier mode inside the persistent kernel
-    void* args[] = {&ka, &noniso, &nic};
+    void* args[] = {&ka, &level, &parent, &noniso, &nic};
     XBFS_CUDA(g, cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(kPersistThreads), args, smem, g->stream));
     return XBFS_OK;
 }
@@ -1537,7 +1579,7 @@ static xbfs_status run_impl(xbfs_graph* g, int64_t source, int32_t* level, int32
     P.st = stats;
     if (use_persist) {
         XBFS_CUDA(g, cudaEventRecord(g->ev0, g->stream));
-        XBFS_TRY(launch_persist(g, a, o.lookahead != 0));
+        XBFS_TRY(launch_persist(g, a, level, parent, o.lookahead != 0));
         XBFS_CUDA(g, cudaEventRecord(g->ev1, g->stream));
     } else if (use_graph) {
         XBFS_CUDA(g, cudaEventRecord(g->ev0, g->stream));
@@ -1570,6 +1612,16 @@ static xbfs_status run_impl(xbfs_graph* g, int64_t source, int32_t* level, int32
         stats->arcs_traversed = hs.arcs_traversed;
         stats->input_edges_traversed = (int64_t)m;
         stats->kernel_launches = hs.launches;
+#if XBFS_BU_PROF
+        {
+            unsigned long long pr[8];
+            cudaMemcpyFromSymbol(pr, g_bu_prof, sizeof(pr));
+            fprintf(stderr, "BUPROF scan %llu first %llu miss %llu hard %llu publish %llu nmiss %llu warps %llu maxwarp %llu\n",
+                    pr[0], pr[1], pr[2], pr[3], pr[4], pr[5], pr[6], pr[7]);
+            memset(pr, 0, sizeof(pr));
+            cudaMemcpyToSymbol(g_bu_prof, pr, sizeof(pr));
+        }
+#endif
         // persistent driver: first CTA entry .. end of init + seed (%globaltimer)
         stats->init_ms = (use_persist && hs.t_enter != ~0ull && hs.t_start >= hs.t_enter)
                              ? (float)((hs.t_start - hs.t_enter) * 1e-6) : 0.f;

@@ -4,6 +4,20 @@
 #pragma once
 #include "common.cuh"
 
+#ifndef XBFS_BU_PROF
+#define XBFS_BU_PROF 0
+#endif
+// dense steps: L2 prefetch of the next group's head32 words (B200 A/B, s24 2x32 roots:
+// 779 with vs 806 GTEPS without: the extra DRAM reads cost more than they hide; off)
+#ifndef XBFS_BU_PF
+#define XBFS_BU_PF 0
+#endif
+// dense chunks: bit-parallel candidate compaction, one store per lane per word (B200 A/B:
+// 815 vs 805 GTEPS)
+#ifndef XBFS_BU_PCOMP
+#define XBFS_BU_PCOMP 1
+#endif
+
 namespace xbfs {
 
 // What a BU step reads and writes.  Vertex indices are LOCAL (the owned range
@@ -21,6 +35,11 @@ struct BuView {
     int* level;                       // owned
     int* parent;                      // owned (global ids)
     int lvl;                          // k + 1
+    unsigned long long* gctr;         // non-NULL: dynamic group scheduling (a zeroed counter of this step)
+    bool dense;                       // a dense step (>= N/16 candidates): prefetch the next group's head32
+#if XBFS_BU_PROF
+    unsigned long long* prof;         // profiling build: per-phase cycle counters
+#endif
 };
 
 
@@ -77,21 +96,62 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, Smem& sm, Publish pub
     const long long nchunks = (b.words + kCW - 1) / kCW;
     const long long gw = (blockIdx.x * (long long)blockDim.x + threadIdx.x) >> 5;
     const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
-    // Static chunk order: warp gw takes chunks gw, gw + nw, ... in groups of 4
-    // (32 lanes = 4 chunks x kCW words): one load round trip tells which of the 4
-    // chunks hold candidates, and the next group's words are loaded one group
-    // ahead (only this warp writes them), so chunks without candidates (most of
-    // them in late BU levels) cost no exposed latency.
+    // A group is 4 chunks (32 lanes = 4 chunks x kCW words): chunks gb + j*st, j < 4.
+    // One load round trip tells which of the 4 chunks hold candidates, and the next
+    // group's words are loaded one group ahead, so chunks without candidates (most
+    // of them in late BU levels) cost no exposed latency.
+    //  static (b.gctr == NULL): warp gw takes chunks gw, gw + nw, ... (gb = gw + 4 nw i, st = nw)
+    //  dynamic (dense steps): group q = 4 consecutive chunks (gb = 4q, st = 1); warp gw takes
+    //    q = gw and gw + nw, then indices 2 nw, 2 nw + 1, ... from a step counter, fetched two
+    //    groups ahead so the atomic's round trip hides behind a group's work: no warp idles
+    //    at the step's end while another still holds several dense groups.
     static_assert(kCW == 8, "4 chunks of 8 words per warp load");
-    auto load_group = [&](long long g0) -> unsigned {
-        const long long cc = g0 + (long long)(lane >> 3) * nw;
+    auto load_group = [&](long long gbase, long long gst) -> unsigned {
+        const long long cc = gbase + (long long)(lane >> 3) * gst;
         const long long ww = cc * kCW + (lane & 7);
         return (cc < nchunks && ww < b.words) ? __ldcg(b.visited + ww) : FULL;
     };
-    unsigned grp_next = load_group(gw);
-    for (long long g0 = gw; g0 < nchunks; g0 += 4 * nw) {
+    const bool dyn = b.gctr != nullptr;
+    const long long st = dyn ? 1 : nw;
+    long long gb = dyn ? 4 * gw : gw;
+    long long q_nxt = gw + nw;                 // dynamic: the group after the current one
+    unsigned grp_next = load_group(gb, st);
+    unsigned grp_nn = dyn ? load_group(4 * q_nxt, 1) : FULL;
+    unsigned long long a2 = 0;                  // dynamic: counter ticket of the group after q_nxt
+    auto advance = [&]() {
+        if (dyn) {
+            gb = 4 * q_nxt;
+            q_nxt = 2 * nw + (long long)__shfl_sync(FULL, a2, 0);
+            grp_next = grp_nn;
+            grp_nn = load_group(4 * q_nxt, 1);
+        } else {
+            gb += 4 * nw;
+        }
+    };
+#if XBFS_BU_PROF
+    long long pt[6] = {0, 0, 0, 0, 0, 0};
+    long long tq = clock64();
+#endif
+    for (; gb < nchunks; advance()) {
         const unsigned grp = grp_next;
-        grp_next = load_group(g0 + 4 * nw);
+        if (dyn) {
+            if (lane == 0) a2 = atomicAdd(b.gctr, 1ull);
+        } else {
+            grp_next = load_group(gb + 4 * nw, nw);
+        }
+        if (XBFS_BU_PF && H32 && b.dense) {
+            // the next group's 1024 vertices' first-probe words into L2 (lane: its 32 vertices,
+            // 4 sectors), so its first probes hit L2 instead of DRAM
+            const long long nb = dyn ? 4 * q_nxt : gb + 4 * nw;
+            const long long cc = nb + (long long)(lane >> 3) * st;
+            const long long ww = cc * kCW + (lane & 7);
+            if (cc < nchunks && ww < b.words) {
+                const unsigned* ph = b.head32 + ww * 32;
+#pragma unroll
+                for (int q = 0; q < 4; ++q) asm volatile("prefetch.global.L2 [%0];" ::"l"(ph + 8 * q));
+            }
+        }
+        const long long g0 = gb;
         // A sparse group (<= kCW*32 candidates over its 4 chunks, the late BU levels)
         // runs as ONE batch: one first-probe round trip for all of it instead of one
         // per chunk.  Dense groups run chunk by chunk.
@@ -101,14 +161,14 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, Smem& sm, Publish pub
         unsigned has = whole ? 1u : __ballot_sync(FULL, grp != FULL);   // lanes whose word has a candidate
         for (int j = 0; has; ++j, has >>= (whole ? 1 : 8)) {
             if (!whole && (has & 0xffu) == 0u) continue;
-            const long long c = g0 + (long long)j * nw;
+            const long long c = g0 + (long long)j * st;
             // 1. candidates of the batch's bitmap words: ballot/popc compaction into shared
             //    memory (the paper's count + prefix-sum + queue-write "double scan").
             long long w;
             bool own;
             unsigned vis;
             if (whole) {                 // lane l: word (l & 7) of chunk g0 + (l >> 3) * nw
-                const long long cc = g0 + (long long)(lane >> 3) * nw;
+                const long long cc = g0 + (long long)(lane >> 3) * st;
                 w = cc * kCW + (lane & 7);
                 own = cc < nchunks && w < b.words;
                 vis = own ? grp : FULL;
@@ -123,7 +183,7 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, Smem& sm, Publish pub
                 const long long wv = v >> 5;
                 if (whole) {
                     const long long cv = wv / kCW;
-                    const int jj = (cv >= g0 + nw) + (cv >= g0 + 2 * nw) + (cv >= g0 + 3 * nw);
+                    const int jj = st == 1 ? (int)(cv - g0) : (cv >= g0 + st) + (cv >= g0 + 2 * st) + (cv >= g0 + 3 * st);
                     return jj * kCW + (int)(wv & (kCW - 1));
                 }
                 return (int)(wv - c * kCW);
@@ -140,7 +200,20 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, Smem& sm, Publish pub
             }
             const int total = __shfl_sync(FULL, incl, 31);
             int pos = incl - cnt;
-            for (unsigned bits = cand; bits; bits &= bits - 1) s_list[wib][pos++] = (int)(w * 32 + __ffs(bits) - 1);
+            if (XBFS_BU_PCOMP && !whole) {
+                // dense chunk: word i's candidates are written by the lanes of their bit
+                // positions, one store per lane per word (kCW rounds instead of up to 32
+                // serial ones in the busiest lane)
+#pragma unroll
+                for (int i = 0; i < kCW; ++i) {
+                    const unsigned ci = __shfl_sync(FULL, cand, i);
+                    const int pi = __shfl_sync(FULL, pos, i);
+                    const long long wi = c * kCW + i;
+                    if ((ci >> lane) & 1u) s_list[wib][pi + __popc(ci & lt)] = (int)(wi * 32 + lane);
+                }
+            } else {
+                for (unsigned bits = cand; bits; bits &= bits - 1) s_list[wib][pos++] = (int)(w * 32 + __ffs(bits) - 1);
+            }
             s_found[wib][lane] = 0;
             if constexpr (LA) sm.la[wib][lane] = 0;
             __syncwarp();
@@ -154,6 +227,9 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, Smem& sm, Publish pub
                     la.edges += (unsigned long long)deg;
                 }
             };
+#if XBFS_BU_PROF
+            { const long long t = clock64(); pt[0] += t - tq; tq = t; }
+#endif
             // 2. first probe of every candidate, kBuFirstIlp candidates per lane in flight:
             //    head[v] (deg << 32 | first stored neighbour) is a dense array read in
             //    candidate order, so a hit (the common case after the degree-desc
@@ -227,6 +303,9 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, Smem& sm, Publish pub
                 }
             }
             __syncwarp();
+#if XBFS_BU_PROF
+            { const long long t = clock64(); pt[1] += t - tq; tq = t; pt[5] += nmiss; }
+#endif
             // 3. the misses: lane-per-candidate, kBuBatch arcs per step in stored
             //    order from the second arc on (look-ahead: from the first, whose
             //    F_{k+1} bit pass 1 did not read); a lane that finishes takes the
@@ -309,6 +388,9 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, Smem& sm, Publish pub
                 nhard += __popc(hm);
             }
             __syncwarp();
+#if XBFS_BU_PROF
+            { const long long t = clock64(); pt[2] += t - tq; tq = t; }
+#endif
             // 4. long unresolved rows: the whole warp probes 32 arcs per step, first hit wins
             for (int h = 0; h < nhard; ++h) {
                 const int hv = s_hard[wib][h];
@@ -347,6 +429,9 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, Smem& sm, Publish pub
                 }
             }
             __syncwarp();
+#if XBFS_BU_PROF
+            { const long long t = clock64(); pt[3] += t - tq; tq = t; }
+#endif
             if (own) {
                 const unsigned f = s_found[wib][lane];
                 unsigned lf = 0u;
@@ -354,8 +439,21 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, Smem& sm, Publish pub
                 if (f | lf) publish(w, vis, f, lf);   // zero words are already zero in every replica
             }
             __syncwarp();
+#if XBFS_BU_PROF
+            { const long long t = clock64(); pt[4] += t - tq; tq = t; }
+#endif
         }
     }
+#if XBFS_BU_PROF
+    // per-warp phase cycles: [0] scan+compaction, [1] first probes, [2] miss loop, [3] hard rows,
+    // [4] publish, [5] misses; [6] warps, [7] max warp total (imbalance)
+    if (lane == 0 && b.prof) {
+        long long tot = 0;
+        for (int i = 0; i < 6; ++i) { atomicAdd(b.prof + i, (unsigned long long)pt[i]); if (i < 5) tot += pt[i]; }
+        atomicAdd(b.prof + 6, 1ull);
+        atomicMax(b.prof + 7, (unsigned long long)tot);
+    }
+#endif
 }
 
 }  // namespace xbfs

@@ -138,6 +138,11 @@ __global__ __launch_bounds__(kBuThreads, 4) void k_bu(DArgs a, int k) {
     b.level = a.level;
     b.parent = a.parent;
     b.lvl = k + 1;
+    b.gctr = nullptr;
+    b.dense = false;
+#if XBFS_BU_PROF
+    b.prof = nullptr;
+#endif
     __shared__ BuSmem<kBuThreads / 32> sm;
     BuLa la_unused;
     bu_chunks<kBuThreads / 32, false, false>(b, sm, [&](long long w, unsigned vis, unsigned f, unsigned) {
@@ -903,6 +908,7 @@ xbfs_status xbfs_run_dist(xbfs_graph* g, int64_t source, int32_t* level, int32_t
     long long reached = 0, arcs_tr = 0;
     int strategy = choose(o, d->arcs_global, fsize, 0, fedges, unvisited, -1);
     int k = 0;
+    unsigned launches = 2;            // k_init, k_seed; then per level k_bu or k_items + k_td + k_merge
     const int grid = grid_for(std::max(d->fwords, d->cw) * 4, 148 * 8);
     const int cap = stats ? stats->level_capacity : 0;
     while (fsize > 0) {
@@ -913,6 +919,7 @@ xbfs_status xbfs_run_dist(xbfs_graph* g, int64_t source, int32_t* level, int32_t
             if (stats->unvisited) stats->unvisited[k] = unvisited;
         }
         XBFS_CUDA(g, cudaMemsetAsync(d->acc, 0, sizeof(DAcc), s));
+        launches += strategy == XBFS_BU ? 1 : 3;
         if (strategy == XBFS_BU) {
             k_bu<<<g->num_sms * 5, kBuThreads, 0, s>>>(a, k);
         } else {
@@ -950,7 +957,7 @@ xbfs_status xbfs_run_dist(xbfs_graph* g, int64_t source, int32_t* level, int32_t
         stats->vertices_reached = reached;
         stats->arcs_traversed = arcs_tr;
         stats->input_edges_traversed = m_total;
-        stats->kernel_launches = 0;
+        stats->kernel_launches = launches;
         stats->num_kernels = 0;
         stats->init_ms = 0.f;
     }
