@@ -1168,8 +1168,228 @@ __device__ __forceinline__ void grid_sync(unsigned* ctr, unsigned& epoch) {
     __syncthreads();
 }
 
+// ------------------------------------------- tiny-frontier mode (f3)
+// SURVEY §8(f) f3 inside the persistent driver: while a scan-free level's frontier
+// is tiny (edgesF_k <= kTinyEdges, |F_k| <= kTinyCap), CTA 0 alone runs the
+// consecutive levels with the queue of F_k in SHARED memory and __syncthreads as
+// the level barrier; the other CTAs wait at one grid barrier and reload the
+// selector state CTA 0 leaves behind.  A level then costs its own dependent
+// round trips (col -> claim -> row_ptr) instead of those plus the global queue
+// staging, the grid barrier and the counter read (small levels
+// are dominated by synchronisation).  The bitmap invariant of the level loop is
+// kept without N/8-byte clears: F_{k-1}'s bits are unset from its queue.
+constexpr int kTinyCap = 2048;       // frontier vertices held in shared memory
+constexpr int kTinyMaxDeg = 64;      // graphs up to this max degree run the TINY instantiation
+constexpr int kTinyEdges = 2048;     // frontier arcs: one or two per thread of the 1024-thread CTA
+constexpr int kTinyDbits = 44;       // packed smem counter: count << 44 | degree sum
+// only from level 16 on: many-level graphs (grids, roads: P:L356) gain (B200, 4096^2 grid:
+// 0.570 vs 0.561 GTEPS), while on Kronecker graphs (7-9 levels) the mode's entry and exit
+// cost about what its few tiny levels save (s24 2x48 roots with it from level 0: 788 vs 800)
+constexpr int kTinyMinLevel = 16;
+
+struct TinySmem {
+    int v[2][kTinyCap];
+    long long rs[2][kTinyCap];
+    long long off[2][kTinyCap + 1];  // exclusive prefix of degrees; off[F] = edgesF
+    unsigned long long ctr;
+};
+
+__device__ __forceinline__ bool tiny_gate(const DevState* st, const SelState& s) {
+    return s.k >= kTinyMinLevel && s.strategy == XBFS_SF && s.queue_valid && st->small_edges > 0 &&
+           s.fedges <= kTinyEdges &&
+           s.fedges <= st->small_edges && s.fsize <= kTinyCap;
+}
+
+// CTA 0 only (blockDim = kPersistThreads).  Entry: F_k in the global queue slot k%3.
+// Exit (the gate fails or the BFS ends): the unexpanded F_k back in slot k%3, every
+// other counter slot zeroed, the selector state stored for the other CTAs.
+__device__ void tiny_levels(const KArgs& a, SelState& s, TinySmem& tm, int* __restrict__ level,
+                            int* __restrict__ parent) {
+    DevState* st = a.st;
+    const int tid = threadIdx.x, lane = tid & 31;
+    const unsigned lt = (1u << lane) - 1u;
+    constexpr int NT = kPersistThreads;
+    int k = s.k;
+    int c = 0;
+    {   // load F_k into buffer 0
+        const int in = k % 3;
+        const long long F = s.fsize;
+        for (long long j = tid; j < F; j += NT) {
+            tm.v[0][j] = __ldcg(a.qv[in] + j);
+            const long long o = __ldcg(a.qoff[in] + j);
+            tm.off[0][j] = o;
+            tm.rs[0][j] = o + __ldcg(a.qdelta[in] + j);
+        }
+        if (tid == 0) tm.off[0][F] = s.fedges;
+        // the stale map fb[(k+2)%3] holds F_{k-1}: unset from its queue (a top-down level
+        // leaves it in slot (k+2)%3), else clear it whole (after a bottom-up level)
+        if (k > 0) {
+            unsigned* stale = a.fb[(k + 2) % 3];
+            if (s.prev_strategy != XBFS_BU && s.fprev <= 8 * kTinyCap) {
+                const int* pq = a.qv[(k + 2) % 3];
+                for (long long j = tid; j < s.fprev; j += NT) {
+                    const int v = __ldcg(pq + j);
+                    atomicAnd(stale + (v >> 5), ~(1u << (v & 31)));
+                }
+            } else {
+                uint4* z4 = reinterpret_cast<uint4*>(stale);
+                for (long long i = tid; i < a.words / 4; i += NT) z4[i] = make_uint4(0, 0, 0, 0);
+                for (long long i = a.words / 4 * 4 + tid; i < a.words; i += NT) stale[i] = 0;
+            }
+        }
+    }
+    __syncthreads();
+    for (;;) {
+        const long long F = s.fsize, T = s.fedges;
+        const int lvl = k + 1;
+        unsigned int* next = a.fb[(k + 1) % 3];
+        if (tid == 0) tm.ctr = 0;
+        __syncthreads();
+        // expand: arc a of F_k owned by the last j with off[j] <= a (binary search in smem)
+        constexpr int R = kTinyEdges / NT;
+        bool win[R];
+        int v[R], u[R];
+        long long rs[R], deg[R];
+#pragma unroll
+        for (int i = 0; i < R; ++i) {
+            const long long arc = tid + (long long)i * NT;
+            v[i] = -1;
+            u[i] = 0;
+            if (arc < T) {
+                int lo = 0, hi = (int)F - 1;
+                while (lo < hi) {
+                    const int mid = (lo + hi + 1) >> 1;
+                    if (tm.off[c][mid] <= arc) lo = mid; else hi = mid - 1;
+                }
+                u[i] = tm.v[c][lo];
+                v[i] = __ldg(a.col + tm.rs[c][lo] + (arc - tm.off[c][lo]));
+            }
+        }
+        unsigned old[R];
+#pragma unroll
+        for (int i = 0; i < R; ++i) old[i] = v[i] >= 0 ? atomicOr(a.visited + (v[i] >> 5), 1u << (v[i] & 31)) : ~0u;
+#pragma unroll
+        for (int i = 0; i < R; ++i) {
+            win[i] = v[i] >= 0 && !((old[i] >> (v[i] & 31)) & 1u);
+            rs[i] = 0;
+            deg[i] = 0;
+            if (win[i]) {
+                level[v[i]] = lvl;
+                parent[v[i]] = u[i];
+                atomicOr(next + (v[i] >> 5), 1u << (v[i] & 31));
+                rs[i] = a.row_ptr[v[i]];
+                deg[i] = a.row_ptr[v[i] + 1];
+            }
+        }
+        // warp-aggregated append to the shared next queue: one smem atomic per warp on the
+        // packed (count, degree sum) counter gives slots and exact degree offsets
+        int cnt = 0;
+        long long dsum = 0;
+#pragma unroll
+        for (int i = 0; i < R; ++i) {
+            deg[i] -= rs[i];
+            if (win[i]) { ++cnt; dsum += deg[i]; }
+        }
+        if (__any_sync(FULL, cnt > 0)) {
+            int ic = cnt;
+            long long id = dsum;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const int tc = __shfl_up_sync(FULL, ic, o);
+                const long long td = __shfl_up_sync(FULL, id, o);
+                if (lane >= o) { ic += tc; id += td; }
+            }
+            const int wc = __shfl_sync(FULL, ic, 31);
+            const long long wd = __shfl_sync(FULL, id, 31);
+            unsigned long long base = 0;
+            if (lane == 31) base = atomicAdd(&tm.ctr, ((unsigned long long)wc << kTinyDbits) + (unsigned long long)wd);
+            base = __shfl_sync(FULL, base, 31);
+            int slot = (int)(base >> kTinyDbits) + ic - cnt;
+            long long off = (long long)(base & ((1ull << kTinyDbits) - 1ull)) + id - dsum;
+#pragma unroll
+            for (int i = 0; i < R; ++i) {
+                if (!win[i]) continue;
+                tm.v[c ^ 1][slot] = v[i];
+                tm.rs[c ^ 1][slot] = rs[i];
+                tm.off[c ^ 1][slot] = off;
+                ++slot;
+                off += deg[i];
+            }
+        }
+        (void)lt;
+        __syncthreads();
+        const unsigned long long q = tm.ctr;
+        const long long nf = (long long)(q >> kTinyDbits), ne = (long long)(q & ((1ull << kTinyDbits) - 1ull));
+        // F_k's bits leave fb[k%3] now (nobody reads F_k's map at level k+1; it is that level's stale map)
+        for (long long j = tid; j < F; j += NT) {
+            const int w = tm.v[c][j];
+            atomicAnd(a.fb[k % 3] + (w >> 5), ~(1u << (w & 31)));
+        }
+        if (tid == 0) {
+            tm.off[c ^ 1][nf] = ne;
+            if (k < kLogCap) {
+                LevelRec r;
+                r.fsize = F;
+                r.fedges = T;
+                r.unvisited = s.unvisited;
+                r.probes = 0;
+                r.la_found = 0;
+                r.strategy = XBFS_SF;
+                r.pad = 0;
+                r.t_ns = globaltimer();
+                a.log[k] = r;
+            }
+            s.reached += F;
+            s.arcs_traversed += T;
+            s.fprev = F;
+            s.fsize = nf;
+            s.fedges = ne;
+            s.unvisited -= nf;
+            s.prev_strategy = XBFS_SF;
+            s.prev_small = 0;
+            s.queue_valid = 1;
+            s.k = k + 1;
+            if (nf == 0) {
+                s.done = 1;
+                s.nlevels = k + 1;
+            } else {
+                s.strategy = choose_strategy(st, a.arcs, nf, F, ne, s.unvisited, XBFS_SF);
+            }
+        }
+        __syncthreads();
+        k = s.k;
+        c ^= 1;
+        if (s.done || !tiny_gate(st, s)) break;
+    }
+    // exit: the unexpanded F_k (buffer c) into the global queue slot k%3 for the level kernels
+    if (!s.done) {
+        const int ob = k % 3;
+        const long long F = s.fsize;
+        for (long long j = tid; j < F; j += NT) {
+            const long long o = tm.off[c][j], d = tm.off[c][j + 1] - o;
+            a.qv[ob][j] = tm.v[c][j];
+            a.qoff[ob][j] = o;
+            a.qdelta[ob][j] = tm.rs[c][j] - o;
+            if (d > 0) {
+                const long long t0 = (o + kTile - 1) / kTile, t1 = (o + d - 1) / kTile;
+                for (long long t = t0; t <= t1; ++t) a.tile_first[ob][t] = (int)j;
+            }
+        }
+    }
+    if (tid == 0) {
+        for (int i = 0; i < 3; ++i) {
+            st->qctr[i] = i == k % 3 ? ((unsigned long long)s.fsize << a.dbits) + (unsigned long long)s.fedges : 0ull;
+            st->qmax[i] = 0;
+            st->acc_found[i] = st->acc_edges[i] = st->acc_probes[i] = st->acc_zero[i] = st->bu_gctr[i] = 0;
+            st->acc_la_found[i] = st->acc_la_edges[i] = 0;
+        }
+        sel_store(st, s);
+    }
+}
+
 template <bool LA>
 union PersistSmem {
+    TinySmem tiny;
     TdSmemT<(XBFS_SS_TPT > XBFS_SF_TPT ? XBFS_SS_TPT : XBFS_SF_TPT)> td;
     typename std::conditional<LA, BuSmemLa<kPersistThreads / 32>, BuSmem<kPersistThreads / 32>>::type bu;
 };
@@ -1179,7 +1399,11 @@ union PersistSmem {
 // DIR: directed graph (f4, reading R-9; also a separate instantiation).
 // (level / parent are kernel parameters here, not loads from the state: parameters
 // live in the constant bank, registers would be held across the whole kernel)
-template <bool LA, bool DIR>
+// TINY: the tiny-frontier mode is a separate instantiation, launched for graphs whose
+// max degree is <= kTinyMaxDeg (grids, road-like graphs: the many-level ones); its mere
+// presence in the Kronecker kernel cost 2.5 % (B200 A/B s24 2x48 roots: 788 vs 808
+// GTEPS, code layout) although it never triggers there.
+template <bool LA, bool DIR, bool TINY = false>
 __global__ __launch_bounds__(kPersistThreads, kPersistBlocks) void k_persist(
     KArgs a, int* __restrict__ level, int* __restrict__ parent, const unsigned int* __restrict__ nonisolated,
     long long nonisolated_count) {
@@ -1201,6 +1425,14 @@ __global__ __launch_bounds__(kPersistThreads, kPersistBlocks) void k_persist(
     for (;;) {
         const int k = s.k, strat = s.strategy, qvalid = s.queue_valid;
         if (s.done) break;
+        if (TINY && !LA && !DIR && tiny_gate(a.st, s)) {
+            // tiny-frontier mode (f3): CTA 0 runs the levels, the others wait here once
+            if (blockIdx.x == 0) tiny_levels(a, s, sm.tiny, level, parent);
+            grid_sync(bar, epoch);
+            if (threadIdx.x == 0 && blockIdx.x != 0) sel_load(a.st, s);
+            __syncthreads();
+            continue;
+        }
         if (blockIdx.x == 0 && threadIdx.x == 0) {
             // slots nobody touches during level k (see select_body)
             a.st->qctr[(k + 2) % 3] = 0;
@@ -1474,11 +1706,13 @@ xbfs_status build_loop_graph(xbfs_graph* g) {
 }
 
 xbfs_status launch_persist(xbfs_graph* g, const KArgs& a, int* level, int* parent, bool lookahead) {
-    static int occ[3][64];
-    static bool init[3][64] = {{false}};
-    const int dev = g->device & 63, v = lookahead ? 1 : (g->directed ? 2 : 0);
+    static int occ[4][64];
+    static bool init[4][64] = {{false}};
+    const bool tiny = !lookahead && !g->directed && g->max_deg <= kTinyMaxDeg;
+    const int dev = g->device & 63, v = lookahead ? 1 : (g->directed ? 2 : (tiny ? 3 : 0));
     void* fn = lookahead ? (void*)k_persist<true, false>
-                         : (g->directed ? (void*)k_persist<false, true> : (void*)k_persist<false, false>);
+                         : (g->directed ? (void*)k_persist<false, true>
+                                        : (tiny ? (void*)k_persist<false, false, true> : (void*)k_persist<false, false>));
     const size_t smem = lookahead ? sizeof(PersistSmem<true>) : sizeof(PersistSmem<false>);
     if (!init[v][dev]) {
         XBFS_CUDA(g, cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
