@@ -70,6 +70,11 @@ def measure(args):
 
 def report(args):
     d = json.load(open(args.report))
+    if args.timing:   # event times from a run outside ncu (same launch sequence)
+        tmg = json.load(open(args.timing))
+        for r, t in zip(d["runs"], tmg["runs"]):
+            assert [x[:2] for x in r["launches"]] == [x[:2] for x in t["launches"]], r["tag"]
+            r["launches"] = t["launches"]
     rows = []
     if args.ncu:
         txt = open(args.ncu).read()
@@ -129,7 +134,7 @@ def report(args):
             hit = e["hit_w"] / e["t"] if e["t"] else float("nan")
             out.append(f"| {k} | {base['fe'][k] / arcs:.3g} | {base['fv'][k]:,} | {sname} | {e['ms']:.4f} | "
                        f"{r['d3'][k] / 1e6:.2f} | {e['dram'] / 1e6:.2f} | {hit:.1f} | "
-                       f"{r['probes'][k]:,} | {'FSB'[base['strategy'][k]] == sname[0]} |")
+                       f"{r['probes'][k]:,} | {'yes' if NAMES[base['strategy'][k]] == sname else ''} |")
         out.append("")
     print("\n".join(out))
 
@@ -141,6 +146,7 @@ def main():
     ap.add_argument("--out", default="gpurun_out/ls.json")
     ap.add_argument("--report", default=None)
     ap.add_argument("--ncu", default=None)
+    ap.add_argument("--timing", default=None, help="JSON of a run outside ncu: its event times are reported")
     args = ap.parse_args()
     if args.report:
         report(args)
