@@ -40,5 +40,16 @@ if os.environ.get("SANITIZE_PERSIST") == "1":
             for opts in (dict(), dict(force_strategy=0), dict(force_strategy=1), dict(force_strategy=2)):
                 g.run(int(root), stats=True, driver=3, **opts)
         g.close()
+# SANITIZE_DIST=1: the multi-GPU path with one rank (build with its peer-memory shuffle, xbfs_run_dist)
+if os.environ.get("SANITIZE_DIST") == "1":
+    from paper_conf_sc_yangls0w24_b200.dist import Comm, DistGraph, xbfs_get_unique_id
+    c = Comm(xbfs_get_unique_id(), 1, 0)
+    for name, (src, dst, n) in {"kron11": synth.kronecker(11, seed=3), "grid": synth.grid(33, 17, seed=1)}.items():
+        dg = DistGraph(c, src, dst, n)
+        for root in synth.roots(n, src, dst, 2, root_seed=4):
+            for opts in (dict(), dict(force_strategy=0), dict(force_strategy=1), dict(force_strategy=2)):
+                dg.run(int(root), **opts)
+        dg.close()
+    c.close()
 torch.cuda.synchronize()
 print("sanitize workload done")
