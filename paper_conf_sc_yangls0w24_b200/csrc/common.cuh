@@ -24,7 +24,10 @@ constexpr int kTile = 2048;          // frontier arcs per td_expand tile
 constexpr int kExpandThreads = 512;  // td_expand block
 constexpr int kBuThreads = 256;      // bu_traverse block (8 warps)
 constexpr int kBuChunkWords = 8;     // bitmap words (256 vertices) per warp chunk
-constexpr int kBuBatch = 8;          // arcs probed per lane step (one 32-byte sector of col)
+#ifndef XBFS_BU_BATCH
+#define XBFS_BU_BATCH 4
+#endif
+constexpr int kBuBatch = XBFS_BU_BATCH;  // arcs probed per lane step (B200 A/B s24: 2 / 3 / 4 / 6 / 8 / 16 -> 796 / 815 / 825 / 822 / 818 / 784 GTEPS)
 #ifndef XBFS_BU_HARD_MIN
 #define XBFS_BU_HARD_MIN 256
 #endif
