@@ -128,6 +128,9 @@ void xbfs_destroy(xbfs_graph* g) {
     for (void* p : dev)
         if (p) cudaFree(p);
     if (g->hctl) cudaFreeHost(g->hctl);
+    if (g->hstage) cudaFreeHost(g->hstage);
+    for (cudaEvent_t e : g->ev_stage)
+        if (e) cudaEventDestroy(e);
     if (g->ev0) cudaEventDestroy(g->ev0);
     if (g->ev1) cudaEventDestroy(g->ev1);
     for (cudaEvent_t e : g->prof_events) cudaEventDestroy(e);

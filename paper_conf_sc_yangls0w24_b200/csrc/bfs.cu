@@ -291,7 +291,7 @@ __device__ __forceinline__ void seed_body(const KArgs& a, int* level, int* paren
     st->fprev = 0;
     st->unvisited = nonisolated_count - (s_cand ? 1 : 0);
     for (int i = 0; i < 3; ++i) {
-        st->acc_found[i] = st->acc_edges[i] = st->acc_probes[i] = st->acc_zero[i] = st->bu_gctr[i] = 0;
+        st->acc_found[i] = st->acc_edges[i] = st->acc_probes[i] = st->acc_zero[i] = 0;
         st->acc_la_found[i] = st->acc_la_edges[i] = 0;
     }
     st->reached = 0;
@@ -442,11 +442,41 @@ __device__ void select_body(const KArgs& a) {
     st->qmax[(k + 2) % 3] = 0;
     st->acc_found[(k + 1) % 3] = st->acc_edges[(k + 1) % 3] = st->acc_probes[(k + 1) % 3] = 0;
     st->acc_zero[(k + 1) % 3] = 0;
-    st->bu_gctr[(k + 1) % 3] = 0;
     st->acc_la_found[(k + 1) % 3] = st->acc_la_edges[(k + 1) % 3] = 0;
     sel_store(st, s);
     mirror_host(a, st);
 }
+
+// Profiling build (XBFS_TL_PROF=1): per level, min / max over CTAs of %globaltimer at
+// the level's start, when the CTA's work is done, after its release fence and when it
+// leaves the level's last barrier; per warp, stamps inside the scan-free expansion of
+// levels < 8 (printed to stderr after a run with stats).
+#ifndef XBFS_TL_PROF
+#define XBFS_TL_PROF 0
+#endif
+#if XBFS_TL_PROF
+constexpr int kTlLevels = 64;
+constexpr int kTlwLevels = 8, kTlwWarps = 8192;
+__device__ unsigned long long g_tl[kTlLevels][4][2];
+__device__ unsigned long long g_tlw[kTlwLevels][5][kTlwWarps];   // SF sub-phases per warp (lane 0)
+__device__ __forceinline__ void tlw_rec(int k, int ph) {
+    const long long gwarp = (blockIdx.x * (long long)blockDim.x + threadIdx.x) >> 5;
+    if ((threadIdx.x & 31) == 0 && k < kTlwLevels && gwarp < kTlwWarps) {
+        unsigned long long t;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+        g_tlw[k][ph][gwarp] = t;
+    }
+}
+__device__ __forceinline__ void tl_rec(int k, int ph, unsigned long long t) {
+    if (k >= 0 && k < kTlLevels) {
+        atomicMin(&g_tl[k][ph][0], t);
+        atomicMax(&g_tl[k][ph][1], t);
+    }
+}
+#define XBFS_TLW(k, ph) tlw_rec(k, ph)
+#else
+#define XBFS_TLW(k, ph) ((void)0)
+#endif
 
 // ----------------------------------------------------------- top-down
 // One tile = kTile consecutive frontier arcs; tile_first gives the first queue
@@ -476,10 +506,32 @@ using TdSmem = TdSmemT<1>;
 #define XBFS_SS_CLAIM 0
 #endif
 
+#ifndef XBFS_SPLIT_MAX
+#define XBFS_SPLIT_MAX 32
+#endif
+constexpr long long kSplitMax = XBFS_SPLIT_MAX;   // parts per base tile when tiles are fewer than CTAs (0: off)
+constexpr long long kSplitMinArcs = 64;            // ... each of at least this many arcs
+
 #ifndef XBFS_SF_PRECHECK_MIN
 #define XBFS_SF_PRECHECK_MIN 65536
 #endif
 constexpr long long kSfPrecheckMin = XBFS_SF_PRECHECK_MIN;   // edgesF_k above which SF probes before claiming
+
+// The top-down probe of visited may go through L1 (XBFS_TD_VIS_L1): within a level the
+// bits only go 0 -> 1, so a stale line can only report a vertex of F_{k+1} as unvisited,
+// which costs SF an atomic that then fails and SS a second store of the same level with
+// another valid parent (C-26); vertices of earlier levels are always seen, because the
+// grid barrier's acquire invalidates L1 (CCTL.IVALL) before every level.
+#ifndef XBFS_TD_VIS_L1
+#define XBFS_TD_VIS_L1 1
+#endif
+__device__ __forceinline__ unsigned ld_vis(const unsigned* p) {
+#if XBFS_TD_VIS_L1
+    return __ldca(p);
+#else
+    return __ldcg(p);
+#endif
+}
 
 // DIR: directed graph (f4, R-9): out-degree-0 winners are counted, not queued.
 template <int MODE, int THREADS, int TPT = 1, bool DIR = false>
@@ -512,12 +564,35 @@ __device__ __forceinline__ void td_expand_body(const KArgs& a, int k, int* __res
     int* s_v = sm.v;
     unsigned lmax = 0;
 
-    const long long nsteps = (ntiles + TPT - 1) / TPT;
+    // Scan-free levels with fewer tiles than CTAs (small frontiers: the first levels, the
+    // tail, many-level graphs): every base tile is split into S equal parts (>= 64 arcs
+    // each; single-scan steps keep whole tiles: B200 A/B s24, its hub level 260 -> 295 us
+    // with the split code in its loop), so that the
+    // scattered claims, stores and row_ptr reads of a small level are spread over up to
+    // every SM instead of queueing in the few that hold a 2048-arc tile (one SM issues
+    // ~1 scattered sector per clock: a tile of winners alone took 7-12 us).
+    const long long nsteps_full = (ntiles + TPT - 1) / TPT;
+    const long long S = (MODE != XBFS_SF || nsteps_full >= gridDim.x || kSplitMax == 0)
+                            ? 0
+                            : max(1LL, min(min((long long)gridDim.x / ntiles, (long long)kSplitMax),
+                                           T / (ntiles * kSplitMinArcs)));
+    const long long nsteps = S ? ntiles * S : nsteps_full;
     for (long long t = blockIdx.x; t < nsteps; t += gridDim.x) {
-        const long long a0 = t * TPT * kTile;
-        const long long a1 = min(a0 + (long long)(TPT * kTile), T);
-        const long long i0 = __ldcg(tfirst + t * TPT);
-        const long long i1 = (t * TPT + TPT < ntiles) ? (long long)__ldcg(tfirst + t * TPT + TPT) : F - 1;
+        long long a0, a1, i0, i1;
+        if (S) {
+            const long long Sd = S > 0 ? S : 1;   // (S == 0 is a compile-time constant for SS)
+            const long long bt = t / Sd, p = t - bt * Sd;
+            const long long b0 = bt * kTile, bl = min(b0 + kTile, T) - b0;
+            a0 = b0 + bl * p / Sd;
+            a1 = b0 + bl * (p + 1) / Sd;
+            i0 = __ldcg(tfirst + bt);
+            i1 = (bt + 1 < ntiles) ? (long long)__ldcg(tfirst + bt + 1) : F - 1;
+        } else {
+            a0 = t * TPT * kTile;
+            a1 = min(a0 + (long long)(TPT * kTile), T);
+            i0 = __ldcg(tfirst + t * TPT);
+            i1 = (t * TPT + TPT < ntiles) ? (long long)__ldcg(tfirst + t * TPT + TPT) : F - 1;
+        }
         const int nv = (int)(i1 - i0 + 1);
         __syncthreads();
         for (int i = threadIdx.x; i < nv; i += THREADS) {
@@ -526,6 +601,7 @@ __device__ __forceinline__ void td_expand_body(const KArgs& a, int k, int* __res
             s_v[i] = __ldcg(qv + i0 + i);
         }
         __syncthreads();
+        if (MODE == XBFS_SF) XBFS_TLW(k, 0);
         // R arcs per thread (stride THREADS: coalesced col reads), processed
         // stage by stage so the R dependent load chains are in flight together.
         constexpr int R = TPT * kTile / THREADS;
@@ -551,7 +627,7 @@ __device__ __forceinline__ void td_expand_body(const KArgs& a, int k, int* __res
             }
         }
 #pragma unroll
-        for (int i = 0; i < R; ++i) vis[i] = !valid[i] ? FULL : (precheck ? __ldcg(visited + (v[i] >> 5)) : 0u);
+        for (int i = 0; i < R; ++i) vis[i] = !valid[i] ? FULL : (precheck ? ld_vis(visited + (v[i] >> 5)) : 0u);
         if (MODE == XBFS_SF) {
             unsigned old[R];
 #pragma unroll
@@ -559,6 +635,15 @@ __device__ __forceinline__ void td_expand_body(const KArgs& a, int k, int* __res
                 const unsigned bit = 1u << (v[i] & 31);
                 old[i] = (vis[i] & bit) ? bit : atomicOr(visited + (v[i] >> 5), bit);
             }
+#if XBFS_TL_PROF
+            {   // stamp once the claims have returned
+                unsigned x = 0;
+#pragma unroll
+                for (int i = 0; i < R; ++i) x |= old[i];
+                if (x == 0x12345678u) __nanosleep(1);
+                XBFS_TLW(k, 1);
+            }
+#endif
 #pragma unroll
             for (int i = 0; i < R; ++i) {
                 const unsigned bit = 1u << (v[i] & 31);
@@ -575,6 +660,7 @@ __device__ __forceinline__ void td_expand_body(const KArgs& a, int k, int* __res
             }
 #pragma unroll
             for (int i = 0; i < R; ++i) deg[i] -= rs[i];
+            XBFS_TLW(k, 2);
             if constexpr (DIR) {
                 int zc = 0;     // winners without out-arcs (directed sinks) are counted, not queued
 #pragma unroll
@@ -587,6 +673,7 @@ __device__ __forceinline__ void td_expand_body(const KArgs& a, int k, int* __res
             }
             enqueue_warp_multi<R>(win, v, rs, deg, &a.st->qctr[(k + 1) % 3], lmax, a.dbits, a.qv[ob],
                                   a.qoff[ob], a.qdelta[ob], a.tile_first[ob]);
+            XBFS_TLW(k, 3);
         } else {
             // single-scan: no status atomics; two threads that both see the bit
             // clear write the same level value (benign race; either parent is
@@ -623,6 +710,7 @@ __device__ __forceinline__ void td_expand_body(const KArgs& a, int k, int* __res
 #endif
         }
     }
+    if (MODE == XBFS_SF) XBFS_TLW(k, 4);
     if (MODE == XBFS_SF && a.track_max) flush_max(&a.st->qmax[(k + 1) % 3], lmax);
 }
 
@@ -767,12 +855,6 @@ __global__ __launch_bounds__(kGenThreads) void k_generate(KArgs a, int role) {
 __device__ unsigned long long g_bu_prof[8];   // profiling build: BU phase cycles of the dense steps
 #endif
 
-// Dynamic group scheduling (bu_core.cuh) for dense steps: at least N/16 candidates.
-// (B200 A/B, s24 2x32 roots: dynamic 752 vs static 788 GTEPS: off by default)
-#ifndef XBFS_BU_DYN
-#define XBFS_BU_DYN 0
-#endif
-
 template <int WARPS, bool LA, class Smem, bool DIR = false>
 __device__ __forceinline__ void bu_body(const KArgs& a, const int* kp, int* __restrict__ level,
                                         int* __restrict__ parent, Smem& sm, bool prefill, long long U) {
@@ -797,8 +879,6 @@ __device__ __forceinline__ void bu_body(const KArgs& a, const int* kp, int* __re
     b.level = level;
     b.parent = parent;
     b.lvl = lvl;
-    b.gctr = (XBFS_BU_DYN && U * 16 >= a.n) ? &a.st->bu_gctr[k % 3] : nullptr;
-    b.dense = U * 16 >= a.n;
 #if XBFS_BU_PROF
     b.prof = U * 16 >= a.n ? g_bu_prof : nullptr;   // the dense steps only
 #endif
@@ -1133,8 +1213,13 @@ __device__ __forceinline__ unsigned ld_acquire(const unsigned* p) {
 // every write of the phase before every read of the next (mutable state is
 // read through L2 everywhere).  A barrier that does not complete within 100 s
 // traps: the run fails with a CUDA error (handle poisoned) instead of hanging.
-__device__ __forceinline__ void grid_sync(unsigned* ctr, unsigned& epoch) {
+__device__ __forceinline__ void grid_sync(unsigned* ctr, unsigned& epoch, int tl = -1) {
     __syncthreads();
+#if XBFS_TL_PROF
+    if (threadIdx.x == 0) tl_rec(tl, 1, globaltimer());
+#else
+    (void)tl;
+#endif
     if (threadIdx.x == 0) {
         ++epoch;
         const unsigned target = epoch * gridDim.x;
@@ -1157,12 +1242,18 @@ __device__ __forceinline__ void grid_sync(unsigned* ctr, unsigned& epoch) {
         asm volatile("fence.acq_rel.gpu;" ::: "memory");
 #else
         __threadfence();
+#if XBFS_TL_PROF
+        tl_rec(tl, 2, globaltimer());
+#endif
         atomicAdd(ctr, 1u);
         if ((int)(ld_acquire(ctr) - target) < 0) {
             const unsigned long long t0 = globaltimer();
             while ((int)(ld_acquire(ctr) - target) < 0)
                 if (globaltimer() - t0 > 100000000000ull) __trap();
         }
+#endif
+#if XBFS_TL_PROF
+        tl_rec(tl, 3, globaltimer());
 #endif
     }
     __syncthreads();
@@ -1380,7 +1471,7 @@ __device__ void tiny_levels(const KArgs& a, SelState& s, TinySmem& tm, int* __re
         for (int i = 0; i < 3; ++i) {
             st->qctr[i] = i == k % 3 ? ((unsigned long long)s.fsize << a.dbits) + (unsigned long long)s.fedges : 0ull;
             st->qmax[i] = 0;
-            st->acc_found[i] = st->acc_edges[i] = st->acc_probes[i] = st->acc_zero[i] = st->bu_gctr[i] = 0;
+            st->acc_found[i] = st->acc_edges[i] = st->acc_probes[i] = st->acc_zero[i] = 0;
             st->acc_la_found[i] = st->acc_la_edges[i] = 0;
         }
         sel_store(st, s);
@@ -1425,6 +1516,9 @@ __global__ __launch_bounds__(kPersistThreads, kPersistBlocks) void k_persist(
     for (;;) {
         const int k = s.k, strat = s.strategy, qvalid = s.queue_valid;
         if (s.done) break;
+#if XBFS_TL_PROF
+        if (threadIdx.x == 0) tl_rec(k, 0, globaltimer());
+#endif
         if (TINY && !LA && !DIR && tiny_gate(a.st, s)) {
             // tiny-frontier mode (f3): CTA 0 runs the levels, the others wait here once
             if (blockIdx.x == 0) tiny_levels(a, s, sm.tiny, level, parent);
@@ -1439,7 +1533,6 @@ __global__ __launch_bounds__(kPersistThreads, kPersistBlocks) void k_persist(
             a.st->qmax[(k + 2) % 3] = 0;
             a.st->acc_found[(k + 1) % 3] = a.st->acc_edges[(k + 1) % 3] = a.st->acc_probes[(k + 1) % 3] = 0;
             a.st->acc_zero[(k + 1) % 3] = 0;
-            a.st->bu_gctr[(k + 1) % 3] = 0;
             a.st->acc_la_found[(k + 1) % 3] = a.st->acc_la_edges[(k + 1) % 3] = 0;
         }
         if (strat != XBFS_BU && !qvalid) {
@@ -1462,7 +1555,7 @@ __global__ __launch_bounds__(kPersistThreads, kPersistBlocks) void k_persist(
             bu_body<kPersistThreads / 32, LA, decltype(sm.bu), DIR>(a, &s.k, level, parent, sm.bu, s.prefill,
                                                                    s.unvisited);
         }
-        grid_sync(bar, epoch);
+        grid_sync(bar, epoch, k);
         if (threadIdx.x == 0) select_step(a, s, blockIdx.x == 0, blockIdx.x == 0 ? globaltimer() : 0ull);
         __syncthreads();
         if (LA && s.la_cf > 0) {    // look-ahead vertices of step k join F_{k+2} before step k+1
@@ -1791,7 +1884,11 @@ static xbfs_status run_impl(xbfs_graph* g, int64_t source, int32_t* level, int32
         return set_error(XBFS_ERR_INVALID_ARG, "lookahead needs the persistent driver (driver 0/3, no plan/profiling)");
     // selection parameters and output pointers live in the device state
     {
-        DevState hs;
+        // a pinned slot whose previous copy has executed (the ring is 4 runs deep)
+        const int slot = g->stage_next;
+        g->stage_next = (slot + 1) % xbfs_graph::kStageSlots;
+        XBFS_CUDA(g, cudaEventSynchronize(g->ev_stage[slot]));
+        DevState& hs = g->hstage[slot];
         memset(&hs, 0, sizeof(hs));
         hs.alpha = o.alpha;
         hs.grow = o.grow;
@@ -1806,6 +1903,7 @@ static xbfs_status run_impl(xbfs_graph* g, int64_t source, int32_t* level, int32
         hs.out_parent = parent;
         hs.t_enter = ~0ull;
         XBFS_CUDA(g, cudaMemcpyAsync(g->st, &hs, sizeof(hs), cudaMemcpyHostToDevice, g->stream));
+        XBFS_CUDA(g, cudaEventRecord(g->ev_stage[slot], g->stream));
     }
     const Grids G = grids_for(g);
     Prof P;
@@ -1846,6 +1944,36 @@ static xbfs_status run_impl(xbfs_graph* g, int64_t source, int32_t* level, int32
         stats->arcs_traversed = hs.arcs_traversed;
         stats->input_edges_traversed = (int64_t)m;
         stats->kernel_launches = hs.launches;
+#if XBFS_TL_PROF
+        {
+            unsigned long long tl[kTlLevels][4][2];
+            cudaMemcpyFromSymbol(tl, g_tl, sizeof(tl));
+            for (int k = 0; k < std::min(hs.nlevels, kTlLevels); ++k) {
+                auto us = [&](unsigned long long t) { return t == ~0ull || t == 0 ? -1.0 : (double)(t - hs.t_start) * 1e-3; };
+                fprintf(stderr, "TL %d start %.2f %.2f done %.2f %.2f fence %.2f %.2f pass %.2f %.2f\n", k,
+                        us(tl[k][0][0]), us(tl[k][0][1]), us(tl[k][1][0]), us(tl[k][1][1]), us(tl[k][2][0]),
+                        us(tl[k][2][1]), us(tl[k][3][0]), us(tl[k][3][1]));
+            }
+            for (int k = 0; k < kTlLevels; ++k)
+                for (int p = 0; p < 4; ++p) { tl[k][p][0] = ~0ull; tl[k][p][1] = 0; }
+            cudaMemcpyToSymbol(g_tl, tl, sizeof(tl));
+            static unsigned long long tw[kTlwLevels][5][kTlwWarps];
+            cudaMemcpyFromSymbol(tw, g_tlw, sizeof(tw));
+            for (int k = 0; k < std::min(hs.nlevels, kTlwLevels); ++k) {
+                fprintf(stderr, "TLW %d", k);
+                for (int p = 0; p < 5; ++p) {
+                    unsigned long long mx = 0;
+                    int arg = -1;
+                    for (int w = 0; w < kTlwWarps; ++w)
+                        if (tw[k][p][w] > mx && tw[k][p][w] >= hs.t_start) { mx = tw[k][p][w]; arg = w; }
+                    fprintf(stderr, " p%d %.2f (w%d)", p, mx ? (double)(mx - hs.t_start) * 1e-3 : -1.0, arg);
+                }
+                fprintf(stderr, "\n");
+            }
+            memset(tw, 0, sizeof(tw));
+            cudaMemcpyToSymbol(g_tlw, tw, sizeof(tw));
+        }
+#endif
 #if XBFS_BU_PROF
         {
             unsigned long long pr[8];

@@ -7,11 +7,6 @@
 #ifndef XBFS_BU_PROF
 #define XBFS_BU_PROF 0
 #endif
-// dense steps: L2 prefetch of the next group's head32 words (B200 A/B, s24 2x32 roots:
-// 779 with vs 806 GTEPS without: the extra DRAM reads cost more than they hide; off)
-#ifndef XBFS_BU_PF
-#define XBFS_BU_PF 0
-#endif
 // dense chunks: bit-parallel candidate compaction, one store per lane per word (B200 A/B:
 // 815 vs 805 GTEPS)
 #ifndef XBFS_BU_PCOMP
@@ -19,6 +14,22 @@
 #endif
 
 namespace xbfs {
+
+// The frontier bitmap F_k is read-only during a BU step: its words are loaded through L1
+// (the first probes of a dense step mostly hit the few words of the hubs).  Safe in the
+// persistent kernel because the grid barrier before the step ends in an acquire load
+// that invalidates the SM's L1 (CCTL.IVALL), and the per-level kernels start with a
+// clean L1.  XBFS_BU_CUR_L1=0: through L2 (ld.cg) as the mutable arrays.
+#ifndef XBFS_BU_CUR_L1
+#define XBFS_BU_CUR_L1 1
+#endif
+__device__ __forceinline__ unsigned ld_cur(const unsigned* p) {
+#if XBFS_BU_CUR_L1
+    return __ldca(p);
+#else
+    return __ldcg(p);
+#endif
+}
 
 // What a BU step reads and writes.  Vertex indices are LOCAL (the owned range
 // starts at 0); col values and the frontier bitmap `cur` are GLOBAL.
@@ -35,8 +46,6 @@ struct BuView {
     int* level;                       // owned
     int* parent;                      // owned (global ids)
     int lvl;                          // k + 1
-    unsigned long long* gctr;         // non-NULL: dynamic group scheduling (a zeroed counter of this step)
-    bool dense;                       // a dense step (>= N/16 candidates): prefetch the next group's head32
 #if XBFS_BU_PROF
     unsigned long long* prof;         // profiling build: per-phase cycle counters
 #endif
@@ -67,8 +76,8 @@ struct BuLa {
 
 // publish(w, vis, found_word, la_word): store the owned word w of F_{k+1} (and of
 // the look-ahead set) and update visited.
-// Mutable state (visited, cur) is read through L2 (__ldcg): the persistent
-// driver runs every level inside one kernel, where L1 lines are not refreshed.
+// Mutable state (visited) is read through L2 (__ldcg); F_k, read-only during the
+// step, through L1 (ld_cur).
 //
 // LA ("since v7 is updated in this phase, v8, which
 // belongs to the next level, can be updated in this bottom-up"): a candidate whose
@@ -96,61 +105,29 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, Smem& sm, Publish pub
     const long long nchunks = (b.words + kCW - 1) / kCW;
     const long long gw = (blockIdx.x * (long long)blockDim.x + threadIdx.x) >> 5;
     const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
-    // A group is 4 chunks (32 lanes = 4 chunks x kCW words): chunks gb + j*st, j < 4.
-    // One load round trip tells which of the 4 chunks hold candidates, and the next
-    // group's words are loaded one group ahead, so chunks without candidates (most
-    // of them in late BU levels) cost no exposed latency.
-    //  static (b.gctr == NULL): warp gw takes chunks gw, gw + nw, ... (gb = gw + 4 nw i, st = nw)
-    //  dynamic (dense steps): group q = 4 consecutive chunks (gb = 4q, st = 1); warp gw takes
-    //    q = gw and gw + nw, then indices 2 nw, 2 nw + 1, ... from a step counter, fetched two
-    //    groups ahead so the atomic's round trip hides behind a group's work: no warp idles
-    //    at the step's end while another still holds several dense groups.
+    // A group is 4 chunks (32 lanes = 4 chunks x kCW words): warp gw takes chunks gb + j*nw,
+    // j < 4, for gb = gw, gw + 4 nw, ...  One load round trip tells which of the 4 chunks
+    // hold candidates, and the next group's words are loaded one group ahead, so chunks
+    // without candidates (most of them in late BU levels) cost no exposed latency.
+    // (B200 A/B, round 2: a balanced contiguous word range per warp instead: s24 -0.8 %,
+    // s20 -1 %; dynamic group scheduling from a step counter: 752 vs 788 GTEPS; an L2
+    // prefetch of the next group's head32: 779 vs 806)
     static_assert(kCW == 8, "4 chunks of 8 words per warp load");
     auto load_group = [&](long long gbase, long long gst) -> unsigned {
         const long long cc = gbase + (long long)(lane >> 3) * gst;
         const long long ww = cc * kCW + (lane & 7);
         return (cc < nchunks && ww < b.words) ? __ldcg(b.visited + ww) : FULL;
     };
-    const bool dyn = b.gctr != nullptr;
-    const long long st = dyn ? 1 : nw;
-    long long gb = dyn ? 4 * gw : gw;
-    long long q_nxt = gw + nw;                 // dynamic: the group after the current one
+    const long long st = nw;
+    long long gb = gw;
     unsigned grp_next = load_group(gb, st);
-    unsigned grp_nn = dyn ? load_group(4 * q_nxt, 1) : FULL;
-    unsigned long long a2 = 0;                  // dynamic: counter ticket of the group after q_nxt
-    auto advance = [&]() {
-        if (dyn) {
-            gb = 4 * q_nxt;
-            q_nxt = 2 * nw + (long long)__shfl_sync(FULL, a2, 0);
-            grp_next = grp_nn;
-            grp_nn = load_group(4 * q_nxt, 1);
-        } else {
-            gb += 4 * nw;
-        }
-    };
 #if XBFS_BU_PROF
     long long pt[6] = {0, 0, 0, 0, 0, 0};
     long long tq = clock64();
 #endif
-    for (; gb < nchunks; advance()) {
+    for (; gb < nchunks; gb += 4 * nw) {
         const unsigned grp = grp_next;
-        if (dyn) {
-            if (lane == 0) a2 = atomicAdd(b.gctr, 1ull);
-        } else {
-            grp_next = load_group(gb + 4 * nw, nw);
-        }
-        if (XBFS_BU_PF && H32 && b.dense) {
-            // the next group's 1024 vertices' first-probe words into L2 (lane: its 32 vertices,
-            // 4 sectors), so its first probes hit L2 instead of DRAM
-            const long long nb = dyn ? 4 * q_nxt : gb + 4 * nw;
-            const long long cc = nb + (long long)(lane >> 3) * st;
-            const long long ww = cc * kCW + (lane & 7);
-            if (cc < nchunks && ww < b.words) {
-                const unsigned* ph = b.head32 + ww * 32;
-#pragma unroll
-                for (int q = 0; q < 4; ++q) asm volatile("prefetch.global.L2 [%0];" ::"l"(ph + 8 * q));
-            }
-        }
+        grp_next = load_group(gb + 4 * nw, nw);
         const long long g0 = gb;
         // A sparse group (<= kCW*32 candidates over its 4 chunks, the late BU levels)
         // runs as ONE batch: one first-probe round trip for all of it instead of one
@@ -187,6 +164,10 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, Smem& sm, Publish pub
                     return jj * kCW + (int)(wv & (kCW - 1));
                 }
                 return (int)(wv - c * kCW);
+            };
+            auto put = [&](int v, int pu) {
+                b.level[v] = b.lvl;
+                b.parent[v] = pu;
             };
             const unsigned cand = ~vis;
             // (chunks without a candidate were skipped above: F_{k+1} words start out
@@ -262,7 +243,7 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, Smem& sm, Publish pub
     #pragma unroll
                 for (int g = 0; g < kBuFirstIlp; ++g) {
                     const int fu = (int)(unsigned)hv[g];
-                    wd[g] = vv[g] >= 0 ? __ldcg(b.cur + (fu >> 5)) : 0u;
+                    wd[g] = vv[g] >= 0 ? ld_cur(b.cur + (fu >> 5)) : 0u;
                     // look-ahead: a degree-1 miss needs its only neighbour's F_{k+1} bit
                     wn[g] = (LA && vv[g] >= 0 && (hv[g] >> 32) == 1) ? __ldcg(b.nxt + (fu >> 5)) : 0u;
                 }
@@ -275,8 +256,7 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, Smem& sm, Publish pub
                         const int fu = (int)(unsigned)hv[g];
                         const long long d = (long long)(hv[g] >> 32);
                         if ((wd[g] >> (fu & 31)) & 1u) {
-                            b.level[v] = b.lvl;
-                            b.parent[v] = fu;
+                            put(v, fu);
                             atomicOr(&s_found[wib][slot(v)], 1u << (v & 31));
                             if (!H32 || (unsigned)d < dmax) {
                                 edges += (unsigned long long)d;
@@ -343,7 +323,7 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, Smem& sm, Publish pub
                     for (int j = 0; j < kBuBatch; ++j) u[j] = (p + j < end) ? __ldg(b.col + p + j) : -1;
     #pragma unroll
                     for (int j = 0; j < kBuBatch; ++j) {
-                        wd[j] = u[j] >= 0 ? __ldcg(b.cur + (u[j] >> 5)) : 0u;
+                        wd[j] = u[j] >= 0 ? ld_cur(b.cur + (u[j] >> 5)) : 0u;
                         wn[j] = (LA && lau < 0 && u[j] >= 0) ? __ldcg(b.nxt + (u[j] >> 5)) : 0u;
                     }
                     int hit = -1;
@@ -359,8 +339,7 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, Smem& sm, Publish pub
                         int pu = u[0];
     #pragma unroll
                         for (int j = 1; j < kBuBatch; ++j) if (j == hit) pu = u[j];
-                        b.level[v] = b.lvl;
-                        b.parent[v] = pu;
+                        put(v, pu);
                         atomicOr(&s_found[wib][slot(v)], 1u << (v & 31));
                         edges += (unsigned long long)(re - rs);
                         fmax = max(fmax, (unsigned)(re - rs));
@@ -401,13 +380,12 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, Smem& sm, Publish pub
                 for (long long base = hrs + s_hoff[wib][h]; base < hre; base += 32) {
                     const long long pp = base + lane;
                     const int u = pp < hre ? __ldg(b.col + pp) : -1;
-                    const bool hit = u >= 0 && ((__ldcg(b.cur + (u >> 5)) >> (u & 31)) & 1u);
+                    const bool hit = u >= 0 && ((ld_cur(b.cur + (u >> 5)) >> (u & 31)) & 1u);
                     const unsigned m = __ballot_sync(FULL, hit);
                     if (m) {
                         const int first = __ffs(m) - 1;
                         if (lane == first) {
-                            b.level[hv] = b.lvl;
-                            b.parent[hv] = u;
+                            put(hv, u);
                             atomicOr(&s_found[wib][slot(hv)], 1u << (hv & 31));
                             edges += (unsigned long long)(hre - hrs);
                             fmax = max(fmax, (unsigned)(hre - hrs));

@@ -277,6 +277,9 @@ xbfs_status alloc_work(xbfs_graph* g) {
     XBFS_CUDA(g, cudaMalloc(&g->red_scratch, 8 * sizeof(unsigned long long)));
     XBFS_CUDA(g, cudaHostAlloc(&g->hctl, sizeof(HostCtl), cudaHostAllocMapped));
     XBFS_CUDA(g, cudaHostGetDevicePointer(&g->hctl_dev, g->hctl, 0));
+    XBFS_CUDA(g, cudaHostAlloc(&g->hstage, xbfs_graph::kStageSlots * sizeof(DevState), cudaHostAllocDefault));
+    for (int i = 0; i < xbfs_graph::kStageSlots; ++i)
+        XBFS_CUDA(g, cudaEventCreateWithFlags(&g->ev_stage[i], cudaEventDisableTiming));
     XBFS_CUDA(g, cudaEventCreate(&g->ev0));
     XBFS_CUDA(g, cudaEventCreate(&g->ev1));
     // The packed queue counter keeps |F| in the high bits and the degree sum in

@@ -84,7 +84,6 @@ struct DevState {
     unsigned long long acc_found[3], acc_edges[3], acc_probes[3];  // BU / SS-count accumulators:
                                  // level k adds into slot k%3; slot (k+1)%3 is zeroed before level k+1
     unsigned long long acc_la_found[3], acc_la_edges[3];  // BU look-ahead (level k+2) discoveries, same slots
-    unsigned long long bu_gctr[3];    // dynamic group counter of a dense BU step, same slots
     unsigned long long acc_zero[3];   // SF winners with out-degree 0 (directed sinks), same slots: counted
                                       // in |F_{k+1}| but never queued (a tile's queue range stays <= its arcs)
     long long reached, arcs_traversed;
@@ -177,6 +176,13 @@ struct xbfs_graph {
     xbfs::LevelRec* log = nullptr;
     xbfs::HostCtl* hctl = nullptr;       // pinned host
     xbfs::HostCtl* hctl_dev = nullptr;   // its device alias
+    // pinned staging ring of the per-run state: the H2D copy that resets the device state
+    // stays asynchronous (from pageable memory the driver may wait for the stream first,
+    // so the launch that follows was issued only once the GPU had gone idle)
+    static constexpr int kStageSlots = 4;
+    xbfs::DevState* hstage = nullptr;
+    cudaEvent_t ev_stage[kStageSlots] = {nullptr, nullptr, nullptr, nullptr};
+    int stage_next = 0;
     unsigned long long* red_scratch = nullptr;  // reductions for stats
     int* scratch_level = nullptr;        // xbfs_run_host device scratch: 2 slots of N (batch pipelining)
     int* scratch_parent = nullptr;
