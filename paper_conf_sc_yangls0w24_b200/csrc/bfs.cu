@@ -182,7 +182,8 @@ __device__ __forceinline__ void mirror_host(const KArgs& a, const DevState* st) 
 // its seed values instead (level 0, parent = itself, visited and F_0 bits), so the
 // seed needs no barrier of its own after the fill.
 __device__ __forceinline__ void init_body(const KArgs& a, int* __restrict__ level, int* __restrict__ parent,
-                                          const unsigned int* __restrict__ nonisolated, long long src = -1) {
+                                          const unsigned int* __restrict__ nonisolated, long long src = -1,
+                                          bool clear_la = false) {
     const long long tid = blockIdx.x * (long long)blockDim.x + threadIdx.x;
     const long long nth = (long long)gridDim.x * blockDim.x;
     const long long n4 = a.n / 4;
@@ -230,7 +231,7 @@ __device__ __forceinline__ void init_body(const KArgs& a, int* __restrict__ leve
         a.fb[0][w] = w == sw ? sbit : 0u;
         a.fb[1][w] = 0;
         a.fb[2][w] = 0;
-        a.la[w] = 0;
+        if (clear_la) a.la[w] = 0;   // (look-ahead map: the LA instantiation only)
     }
 }
 
@@ -291,7 +292,7 @@ __device__ __forceinline__ void seed_body(const KArgs& a, int* level, int* paren
     st->fprev = 0;
     st->unvisited = nonisolated_count - (s_cand ? 1 : 0);
     for (int i = 0; i < 3; ++i) {
-        st->acc_found[i] = st->acc_edges[i] = st->acc_probes[i] = st->acc_zero[i] = 0;
+        st->acc_found[i] = st->acc_edges[i] = st->acc_probes[i] = st->acc_zero[i] = st->td_ctr[i] = 0;
         st->acc_la_found[i] = st->acc_la_edges[i] = 0;
     }
     st->reached = 0;
@@ -442,6 +443,7 @@ __device__ void select_body(const KArgs& a) {
     st->qmax[(k + 2) % 3] = 0;
     st->acc_found[(k + 1) % 3] = st->acc_edges[(k + 1) % 3] = st->acc_probes[(k + 1) % 3] = 0;
     st->acc_zero[(k + 1) % 3] = 0;
+    st->td_ctr[(k + 1) % 3] = 0;
     st->acc_la_found[(k + 1) % 3] = st->acc_la_edges[(k + 1) % 3] = 0;
     sel_store(st, s);
     mirror_host(a, st);
@@ -457,7 +459,7 @@ __device__ void select_body(const KArgs& a) {
 #if XBFS_TL_PROF
 constexpr int kTlLevels = 64;
 constexpr int kTlwLevels = 8, kTlwWarps = 8192;
-__device__ unsigned long long g_tl[kTlLevels][4][2];
+__device__ unsigned long long g_tl[kTlLevels][8][2];   // phases 0-3 last barrier, 5-7 a mid-level one
 __device__ unsigned long long g_tlw[kTlwLevels][5][kTlwWarps];   // SF sub-phases per warp (lane 0)
 __device__ __forceinline__ void tlw_rec(int k, int ph) {
     const long long gwarp = (blockIdx.x * (long long)blockDim.x + threadIdx.x) >> 5;
@@ -492,6 +494,7 @@ struct TdSmemT {
     long long off[TPT * kTile + 1];
     long long delta[TPT * kTile + 1];
     int v[TPT * kTile + 1];
+    long long next;   // dynamic scheduling: the CTA's next step
 };
 using TdSmem = TdSmemT<1>;
 
@@ -506,6 +509,9 @@ using TdSmem = TdSmemT<1>;
 #define XBFS_SS_CLAIM 0
 #endif
 
+#ifndef XBFS_TD_DYN
+#define XBFS_TD_DYN 1
+#endif
 #ifndef XBFS_SPLIT_MAX
 #define XBFS_SPLIT_MAX 32
 #endif
@@ -577,7 +583,16 @@ __device__ __forceinline__ void td_expand_body(const KArgs& a, int k, int* __res
                             : max(1LL, min(min((long long)gridDim.x / ntiles, (long long)kSplitMax),
                                            T / (ntiles * kSplitMinArcs)));
     const long long nsteps = S ? ntiles * S : nsteps_full;
-    for (long long t = blockIdx.x; t < nsteps; t += gridDim.x) {
+    // Large single-scan steps take their steps from a ticket counter instead of
+    // round-robin: the cost of a step varies with how many of its arcs discover a vertex,
+    // and the static deal left the CTAs of a hub level finishing 25-35 us apart (level
+    // timeline, s24).  Thread 0 holds the ticket of the step after next, so the atomic's
+    // round trip hides behind a whole step.
+    const bool dyn = XBFS_TD_DYN && MODE == XBFS_SS && nsteps >= 2 * (long long)gridDim.x;
+    unsigned long long* tctr = &a.st->td_ctr[k % 3];
+    unsigned long long tk = 0;
+    if (dyn && threadIdx.x == 0) tk = gridDim.x + atomicAdd(tctr, 1ull);
+    for (long long t = blockIdx.x; t < nsteps;) {
         long long a0, a1, i0, i1;
         if (S) {
             const long long Sd = S > 0 ? S : 1;   // (S == 0 is a compile-time constant for SS)
@@ -595,12 +610,17 @@ __device__ __forceinline__ void td_expand_body(const KArgs& a, int k, int* __res
         }
         const int nv = (int)(i1 - i0 + 1);
         __syncthreads();
+        if (dyn && threadIdx.x == 0) {
+            sm.next = (long long)tk;
+            tk = gridDim.x + atomicAdd(tctr, 1ull);
+        }
         for (int i = threadIdx.x; i < nv; i += THREADS) {
             s_off[i] = __ldcg(qoff + i0 + i);
             s_delta[i] = __ldcg(qdelta + i0 + i);
             s_v[i] = __ldcg(qv + i0 + i);
         }
         __syncthreads();
+        const long long t_next = dyn ? sm.next : t + gridDim.x;
         if (MODE == XBFS_SF) XBFS_TLW(k, 0);
         // R arcs per thread (stride THREADS: coalesced col reads), processed
         // stage by stage so the R dependent load chains are in flight together.
@@ -709,6 +729,7 @@ __device__ __forceinline__ void td_expand_body(const KArgs& a, int k, int* __res
             }
 #endif
         }
+        t = t_next;
     }
     if (MODE == XBFS_SF) XBFS_TLW(k, 4);
     if (MODE == XBFS_SF && a.track_max) flush_max(&a.st->qmax[(k + 1) % 3], lmax);
@@ -737,20 +758,27 @@ __device__ __forceinline__ void ss_count_body(const KArgs& a, int k) {
         unsigned word = __ldcg(bm + w);
         if (!word) continue;
         found += __popc(word);
-        // up to 8 head[] loads in flight per step (a dense frontier word holds several bits)
+        // up to 8 head32[] loads in flight per step (a dense frontier word holds several
+        // bits); the 4-byte word halves the bytes of the 8-byte head[] (a saturated degree
+        // field, deg >= dmax, falls back to the row_ptr pair)
+        const unsigned dmax = a.idbits >= 32 ? 0u : (0xffffffffu >> a.idbits);
         while (word) {
-            unsigned long long hv[8];
+            unsigned hv[8];
+            int vx[8];
 #pragma unroll
             for (int i = 0; i < 8; ++i) {
-                hv[i] = 0ull;
+                hv[i] = 0u;
+                vx[i] = -1;
                 if (word) {
-                    hv[i] = __ldg(a.head + w * 32 + __ffs(word) - 1);
+                    vx[i] = (int)(w * 32 + __ffs(word) - 1);
+                    hv[i] = __ldg(a.head32 + vx[i]);
                     word &= word - 1;
                 }
             }
 #pragma unroll
             for (int i = 0; i < 8; ++i) {
-                const unsigned d = (unsigned)(hv[i] >> 32);
+                unsigned d = a.idbits >= 32 ? dmax : hv[i] >> a.idbits;
+                if (vx[i] >= 0 && d >= dmax) d = (unsigned)(a.row_ptr[vx[i] + 1] - a.row_ptr[vx[i]]);
                 edges += d;
                 gmax = max(gmax, d);
             }
@@ -1161,7 +1189,7 @@ __global__ void __cluster_dims__(kSmallCluster, 1, 1) __launch_bounds__(kSmallTh
         st->reached = reached;
         st->arcs_traversed = arcs_tr;
         st->prev_strategy = XBFS_SF;
-        for (int i = 0; i < 3; ++i) st->acc_found[i] = st->acc_edges[i] = st->acc_probes[i] = st->acc_zero[i] = 0;
+        for (int i = 0; i < 3; ++i) st->acc_found[i] = st->acc_edges[i] = st->acc_probes[i] = st->acc_zero[i] = st->td_ctr[i] = 0;
         st->fmaxdeg = fmaxdeg;
         st->advanced = st->mirror_host ? 0 : 1;   // graph driver: its k_select node only mirrors
         st->prev_small = 1;
@@ -1213,10 +1241,10 @@ __device__ __forceinline__ unsigned ld_acquire(const unsigned* p) {
 // every write of the phase before every read of the next (mutable state is
 // read through L2 everywhere).  A barrier that does not complete within 100 s
 // traps: the run fails with a CUDA error (handle poisoned) instead of hanging.
-__device__ __forceinline__ void grid_sync(unsigned* ctr, unsigned& epoch, int tl = -1) {
+__device__ __forceinline__ void grid_sync(unsigned* ctr, unsigned& epoch, int tl = -1, int ph0 = 0) {
     __syncthreads();
 #if XBFS_TL_PROF
-    if (threadIdx.x == 0) tl_rec(tl, 1, globaltimer());
+    if (threadIdx.x == 0) tl_rec(tl, ph0 + 1, globaltimer());
 #else
     (void)tl;
 #endif
@@ -1243,7 +1271,7 @@ __device__ __forceinline__ void grid_sync(unsigned* ctr, unsigned& epoch, int tl
 #else
         __threadfence();
 #if XBFS_TL_PROF
-        tl_rec(tl, 2, globaltimer());
+        tl_rec(tl, ph0 + 2, globaltimer());
 #endif
         atomicAdd(ctr, 1u);
         if ((int)(ld_acquire(ctr) - target) < 0) {
@@ -1253,7 +1281,7 @@ __device__ __forceinline__ void grid_sync(unsigned* ctr, unsigned& epoch, int tl
         }
 #endif
 #if XBFS_TL_PROF
-        tl_rec(tl, 3, globaltimer());
+        tl_rec(tl, ph0 + 3, globaltimer());
 #endif
     }
     __syncthreads();
@@ -1471,7 +1499,7 @@ __device__ void tiny_levels(const KArgs& a, SelState& s, TinySmem& tm, int* __re
         for (int i = 0; i < 3; ++i) {
             st->qctr[i] = i == k % 3 ? ((unsigned long long)s.fsize << a.dbits) + (unsigned long long)s.fedges : 0ull;
             st->qmax[i] = 0;
-            st->acc_found[i] = st->acc_edges[i] = st->acc_probes[i] = st->acc_zero[i] = 0;
+            st->acc_found[i] = st->acc_edges[i] = st->acc_probes[i] = st->acc_zero[i] = st->td_ctr[i] = 0;
             st->acc_la_found[i] = st->acc_la_edges[i] = 0;
         }
         sel_store(st, s);
@@ -1507,7 +1535,7 @@ __global__ __launch_bounds__(kPersistThreads, kPersistBlocks) void k_persist(
     count_launch(a.st);
     // the source's entries are written by the fill itself and the seed state by one
     // thread alongside it: one barrier for both
-    init_body(a, level, parent, nonisolated, *(const volatile long long*)&a.st->source);
+    init_body(a, level, parent, nonisolated, *(const volatile long long*)&a.st->source, LA);
     if (blockIdx.x == 0 && threadIdx.x == 0) seed_body(a, level, parent, nonisolated_count, nonisolated, true);
     grid_sync(bar, epoch);
     if (blockIdx.x == 0 && threadIdx.x == 0) a.st->t_start = globaltimer();
@@ -1533,6 +1561,7 @@ __global__ __launch_bounds__(kPersistThreads, kPersistBlocks) void k_persist(
             a.st->qmax[(k + 2) % 3] = 0;
             a.st->acc_found[(k + 1) % 3] = a.st->acc_edges[(k + 1) % 3] = a.st->acc_probes[(k + 1) % 3] = 0;
             a.st->acc_zero[(k + 1) % 3] = 0;
+            a.st->td_ctr[(k + 1) % 3] = 0;
             a.st->acc_la_found[(k + 1) % 3] = a.st->acc_la_edges[(k + 1) % 3] = 0;
         }
         if (strat != XBFS_BU && !qvalid) {
@@ -1548,7 +1577,7 @@ __global__ __launch_bounds__(kPersistThreads, kPersistBlocks) void k_persist(
             td_expand_body<XBFS_SS, kPersistThreads, XBFS_SS_TPT, DIR>(
                 a, k, level, parent, *reinterpret_cast<TdSmemT<XBFS_SS_TPT>*>(&sm.td), DIR ? -1 : s.fsize,
                 s.fedges);
-            grid_sync(bar, epoch);
+            grid_sync(bar, epoch, k, 4);
             ss_count_body(a, k);
         } else {
             // (directed: bu_body sums edgesF_{k+1} over out-arcs itself)
@@ -1946,16 +1975,20 @@ static xbfs_status run_impl(xbfs_graph* g, int64_t source, int32_t* level, int32
         stats->kernel_launches = hs.launches;
 #if XBFS_TL_PROF
         {
-            unsigned long long tl[kTlLevels][4][2];
+            unsigned long long tl[kTlLevels][8][2];
             cudaMemcpyFromSymbol(tl, g_tl, sizeof(tl));
             for (int k = 0; k < std::min(hs.nlevels, kTlLevels); ++k) {
                 auto us = [&](unsigned long long t) { return t == ~0ull || t == 0 ? -1.0 : (double)(t - hs.t_start) * 1e-3; };
-                fprintf(stderr, "TL %d start %.2f %.2f done %.2f %.2f fence %.2f %.2f pass %.2f %.2f\n", k,
+                fprintf(stderr, "TL %d start %.2f %.2f done %.2f %.2f fence %.2f %.2f pass %.2f %.2f", k,
                         us(tl[k][0][0]), us(tl[k][0][1]), us(tl[k][1][0]), us(tl[k][1][1]), us(tl[k][2][0]),
                         us(tl[k][2][1]), us(tl[k][3][0]), us(tl[k][3][1]));
+                if (tl[k][5][1])
+                    fprintf(stderr, " | mid done %.2f %.2f fence %.2f %.2f pass %.2f %.2f", us(tl[k][5][0]),
+                            us(tl[k][5][1]), us(tl[k][6][0]), us(tl[k][6][1]), us(tl[k][7][0]), us(tl[k][7][1]));
+                fprintf(stderr, "\n");
             }
             for (int k = 0; k < kTlLevels; ++k)
-                for (int p = 0; p < 4; ++p) { tl[k][p][0] = ~0ull; tl[k][p][1] = 0; }
+                for (int p = 0; p < 8; ++p) { tl[k][p][0] = ~0ull; tl[k][p][1] = 0; }
             cudaMemcpyToSymbol(g_tl, tl, sizeof(tl));
             static unsigned long long tw[kTlwLevels][5][kTlwWarps];
             cudaMemcpyFromSymbol(tw, g_tlw, sizeof(tw));

@@ -84,6 +84,7 @@ struct DevState {
     unsigned long long acc_found[3], acc_edges[3], acc_probes[3];  // BU / SS-count accumulators:
                                  // level k adds into slot k%3; slot (k+1)%3 is zeroed before level k+1
     unsigned long long acc_la_found[3], acc_la_edges[3];  // BU look-ahead (level k+2) discoveries, same slots
+    unsigned long long td_ctr[3];     // step tickets of a dynamically scheduled top-down step, same slots
     unsigned long long acc_zero[3];   // SF winners with out-degree 0 (directed sinks), same slots: counted
                                       // in |F_{k+1}| but never queued (a tile's queue range stays <= its arcs)
     long long reached, arcs_traversed;
