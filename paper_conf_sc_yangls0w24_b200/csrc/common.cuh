@@ -33,9 +33,9 @@ constexpr int kBuBatch = XBFS_BU_BATCH;  // arcs probed per lane step (B200 A/B 
 #endif
 constexpr int kBuHardMin = XBFS_BU_HARD_MIN;  // unresolved rows with more arcs left go warp-cooperative
 #ifndef XBFS_BU_FIRST_ILP
-#define XBFS_BU_FIRST_ILP 4
+#define XBFS_BU_FIRST_ILP 5
 #endif
-constexpr int kBuFirstIlp = XBFS_BU_FIRST_ILP;  // first probes in flight per lane
+constexpr int kBuFirstIlp = XBFS_BU_FIRST_ILP;  // first probes in flight per lane (B200 A/B s24 48 roots, round 2: 4 / 5 / 6 -> 826 / 830 / 825 GTEPS)
 constexpr int kGenThreads = 256;
 constexpr int kSmallThreads = 512;   // small-frontier cluster kernel: threads per CTA
 constexpr int kSmallCluster = 8;     // CTAs per cluster (portable size)
