@@ -513,10 +513,13 @@ using TdSmem = TdSmemT<1>;
 #define XBFS_TD_DYN 1
 #endif
 #ifndef XBFS_SPLIT_MAX
-#define XBFS_SPLIT_MAX 32
+#define XBFS_SPLIT_MAX 4
 #endif
-constexpr long long kSplitMax = XBFS_SPLIT_MAX;   // parts per base tile when tiles are fewer than CTAs (0: off)
-constexpr long long kSplitMinArcs = 64;            // ... each of at least this many arcs
+constexpr long long kSplitMax = XBFS_SPLIT_MAX;   // parts per base tile when tiles are fewer than CTAs (0: off; B200 A/B grid 4096^2: 2 / 4 / 8 / 32 -> 0.627 / 0.656 / 0.645 / 0.600 GTEPS, s20 and s24 flat)
+#ifndef XBFS_SPLIT_MIN_ARCS
+#define XBFS_SPLIT_MIN_ARCS 64
+#endif
+constexpr long long kSplitMinArcs = XBFS_SPLIT_MIN_ARCS;            // ... each of at least this many arcs
 
 #ifndef XBFS_SF_PRECHECK_MIN
 #define XBFS_SF_PRECHECK_MIN 65536
