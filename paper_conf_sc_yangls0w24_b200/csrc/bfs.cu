@@ -534,6 +534,11 @@ constexpr long long kSfPrecheckMin = XBFS_SF_PRECHECK_MIN;   // edgesF_k above w
 #ifndef XBFS_TD_VIS_L1
 #define XBFS_TD_VIS_L1 1
 #endif
+// (SS: a vertex found earlier in the same level is seen as visited only through L2, where
+// the REDs land; a stale L1 line costs four scattered writes)
+#ifndef XBFS_SS_VIS_L1
+#define XBFS_SS_VIS_L1 0
+#endif
 __device__ __forceinline__ unsigned ld_vis(const unsigned* p) {
 #if XBFS_TD_VIS_L1
     return __ldca(p);
@@ -650,7 +655,11 @@ __device__ __forceinline__ void td_expand_body(const KArgs& a, int k, int* __res
             }
         }
 #pragma unroll
-        for (int i = 0; i < R; ++i) vis[i] = !valid[i] ? FULL : (precheck ? ld_vis(visited + (v[i] >> 5)) : 0u);
+        for (int i = 0; i < R; ++i)
+            vis[i] = !valid[i] ? FULL
+                               : (!precheck ? 0u
+                                            : ((MODE == XBFS_SF || XBFS_SS_VIS_L1) ? ld_vis(visited + (v[i] >> 5))
+                                                                                   : __ldcg(visited + (v[i] >> 5))));
         if (MODE == XBFS_SF) {
             unsigned old[R];
 #pragma unroll

@@ -49,7 +49,7 @@ int main() {
     cudaStream_t s;
     cudaStreamCreate(&s);
     unsigned epoch = 0;
-    struct V { const char* name; int smem; bool coop; bool fill; bool sync_before; };
+    struct V { const char* name; int smem; bool coop; bool fill; bool sync_before; int grid = 0; int block = 1024; };
     V vs[] = {
         {"coop smem105K, fill, host sync before", 105 << 10, true, true, true},
         {"coop smem105K, fill, no host sync", 105 << 10, true, true, false},
@@ -57,6 +57,9 @@ int main() {
         {"coop smem16, fill, no host sync", 16, true, true, false},
         {"plain smem105K, fill, no host sync", 105 << 10, false, true, false},
         {"plain smem16, fill, no host sync", 16, false, true, false},
+        {"plain 148x256 smem16", 16, false, true, false, 0, 256},
+        {"plain 74x1024 smem16", 16, false, true, false, 74, 1024},
+        {"plain 1x32 (no barrier work)", 16, false, true, false, 1, 32},
     };
     cudaFuncSetAttribute(k_coop, cudaFuncAttributeMaxDynamicSharedMemorySize, 110 << 10);
     for (const V& v : vs) {
@@ -67,11 +70,14 @@ int main() {
             cudaMemcpyToSymbol(g_t, init, sizeof(init));
             if (v.fill) k_fill<<<nsm * 4, 512, 0, s>>>(buf, fill_bytes / 16);
             if (v.sync_before) cudaStreamSynchronize(s);
+            const unsigned zero = 0;
+            cudaMemcpyToSymbolAsync(g_bar, &zero, sizeof(zero), 0, cudaMemcpyHostToDevice, s);
             cudaEventRecord(e0, s);
-            ++epoch;
+            epoch = 1;
             void* args[] = {&epoch};
-            if (v.coop) cudaLaunchCooperativeKernel((void*)k_coop, nsm, 1024, args, v.smem, s);
-            else k_coop<<<nsm, 1024, v.smem, s>>>(epoch);
+            const int gridn = v.grid ? v.grid : nsm;
+            if (v.coop) cudaLaunchCooperativeKernel((void*)k_coop, gridn, v.block, args, v.smem, s);
+            else k_coop<<<gridn, v.block, v.smem, s>>>(epoch);
             cudaEventRecord(e1, s);
             cudaStreamSynchronize(s);
             float ms;

@@ -77,16 +77,16 @@ def main():
     lp = os.path.join(src, "launches.csv")
     if os.path.exists(lp):
         agg = launches(lp)
-        tot_bfs = sum(t for k, (n, t) in agg.items() if not k.startswith(("cub::", "at::")) and "reorder" not in k
-                      and "check_and_pack" not in k and "split_keys" not in k and "degree_facts" not in k
-                      and "count_m" not in k)
+        def is_bfs(k):   # the library's BFS kernels (not the CSR build, stats, CUB / torch validation kernels)
+            return k.startswith("k_") and all(s not in k for s in (
+                "reorder", "check_and_pack", "split_keys", "degree_facts", "count_m", "k_head"))
+        tot_bfs = sum(t for k, (n, t) in agg.items() if is_bfs(k))
         lines += ["## Launch list (`ncu --metrics gpu__time_duration.sum --clock-control none`)", "",
                   "Cold-cache, serialised per-launch times: compare SHARES, not absolutes.  `share` is of the BFS",
                   "kernels only (CSR build / reorder / stats / torch fill kernels excluded).", "",
                   "| kernel | launches | total us | avg us | share of BFS |", "|---|---|---|---|---|"]
         for k, (n, t) in sorted(agg.items(), key=lambda x: -x[1][1]):
-            bfs = not k.startswith(("cub::", "at::")) and all(s not in k for s in (
-                "reorder", "check_and_pack", "split_keys", "degree_facts", "count_m", "k_head"))
+            bfs = is_bfs(k)
             share = f"{100 * t / tot_bfs:.1f}%" if bfs and tot_bfs else "-"
             lines.append(f"| `{k}` | {n} | {t:.1f} | {t / n:.2f} | {share} |")
         lines.append("")
