@@ -138,7 +138,7 @@ def test_kronecker_s20_adaptive(xb):
     g = xb.Graph(_dev(src), _dev(dst), n)
     for root in synth.roots(n, src, dst, 8, root_seed=2):
         st = _check_run(g, og, src, dst, root)
-        assert 2 in st.strategy     # a BU level happens on Kronecker s20 with alpha 0.1
+        assert 2 in st.strategy     # a BU level happens on Kronecker s20 with the default alpha (0.04)
     for root in synth.roots(n, src, dst, 2, root_seed=9):
         for f in (0, 1, 2):
             _check_run(g, og, src, dst, root, force_strategy=f)
@@ -337,10 +337,11 @@ def test_persistent_driver_level_times(xb):
     g.close()
 
 
-def test_deep_levels_escape_the_level_store(xb):
-    """A path deeper than the 2-byte status array (kLvMax = 65533 levels): the
-    deep levels go straight to level[] and the epilogue keeps them; parents
-    below and above the limit are found from mixed entries."""
+def test_deep_path_beyond_the_level_log(xb):
+    """A path of 65,600 levels, deeper than the device's per-level log (kLogCap =
+    65,536 entries) and than any 16-bit level encoding: levels and parents stay
+    exact past the log's end, for the persistent (adaptive, forced BU / SS) and
+    host-loop drivers and a source in the middle."""
     n = 65_600
     src = np.arange(n - 1, dtype=np.uint32)
     dst = src + 1
@@ -354,8 +355,9 @@ def test_deep_levels_escape_the_level_store(xb):
 
 
 def test_unaligned_output_arrays(xb):
-    """The epilogue writes 16-byte groups only when both outputs are 16-byte
-    aligned; offset views take the scalar path and still get every element."""
+    """The init fill writes 32-byte groups only when both outputs are 32-byte
+    aligned (else 16-byte groups, else scalars); offset views of odd length
+    still get every element right."""
     src, dst, n = synth.kronecker(11, seed=9)
     n += 3                                   # N not a multiple of 4; 3 isolated vertices
     og = oracle.build_csr(n, src, dst)
