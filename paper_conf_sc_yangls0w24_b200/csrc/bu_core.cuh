@@ -166,8 +166,8 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, Smem& sm, Publish pub
                 return (int)(wv - c * kCW);
             };
             auto put = [&](int v, int pu) {
-                b.level[v] = b.lvl;
-                b.parent[v] = pu;
+                st_out(b.level + v, b.lvl);
+                st_out(b.parent + v, pu);
             };
             const unsigned cand = ~vis;
             // (chunks without a candidate were skipped above: F_{k+1} words start out
@@ -233,7 +233,7 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, Smem& sm, Publish pub
                     // degree stays dmax (>= 2) and is resolved in pass 3 on a hit
     #pragma unroll
                     for (int g = 0; g < kBuFirstIlp; ++g) {
-                        const unsigned h = vv[g] >= 0 ? __ldg(b.head32 + vv[g]) : 0u;
+                        const unsigned h = vv[g] >= 0 ? ld_ro32<1>(b.head32 + vv[g]) : 0u;
                         hv[g] = ((unsigned long long)(b.idbits >= 32 ? 0u : (h >> b.idbits)) << 32) | (h & idmask);
                     }
                 } else {
@@ -305,8 +305,8 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, Smem& sm, Publish pub
                             fmax = max(fmax, (unsigned)dd);
                             v = -1;
                         } else {
-                            rs = b.row_ptr[v];
-                            re = b.row_ptr[v + 1];
+                            rs = ld_ro64<4>(b.row_ptr + v);
+                            re = ld_ro64<4>(b.row_ptr + v + 1);
                             p = LA ? rs : rs + 1;
                             lau = -1;
                         }
@@ -320,7 +320,7 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, Smem& sm, Publish pub
                     int u[kBuBatch];
                     unsigned wd[kBuBatch], wn[kBuBatch];
     #pragma unroll
-                    for (int j = 0; j < kBuBatch; ++j) u[j] = (p + j < end) ? __ldg(b.col + p + j) : -1;
+                    for (int j = 0; j < kBuBatch; ++j) u[j] = (p + j < end) ? ld_ro32<2>(b.col + p + j) : -1;
     #pragma unroll
                     for (int j = 0; j < kBuBatch; ++j) {
                         wd[j] = u[j] >= 0 ? ld_cur(b.cur + (u[j] >> 5)) : 0u;

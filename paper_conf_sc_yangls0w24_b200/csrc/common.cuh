@@ -20,6 +20,59 @@
 
 namespace xbfs {
 
+// L2 eviction-priority hints (B200 A/B, round 2): the outputs' lines are kept in L2 so
+// the scattered level / parent stores of the levels merge there instead of costing a
+// DRAM read-modify-write; streaming CSR reads may be marked evict-first.
+#ifndef XBFS_OUT_KEEP
+#define XBFS_OUT_KEEP 0
+#endif
+#ifndef XBFS_STREAM_HINT
+#define XBFS_STREAM_HINT 0      // bit 0: head32, bit 1: col, bit 2: row_ptr -> L2 evict_first
+#endif
+__device__ __forceinline__ unsigned long long l2_policy_last() {
+    unsigned long long p;
+    asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ unsigned long long l2_policy_first() {
+    unsigned long long p;
+    asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+// an output store (level / parent)
+__device__ __forceinline__ void st_out(int* p, int v) {
+#if XBFS_OUT_KEEP
+    asm volatile("st.global.L2::cache_hint.b32 [%0], %1, %2;" ::"l"(p), "r"(v), "l"(l2_policy_last()) : "memory");
+#else
+    *p = v;
+#endif
+}
+// read-only streaming loads: head32 (bit 0), col (bit 1), row_ptr (bit 2)
+template <int BIT>
+__device__ __forceinline__ unsigned ld_ro32(const unsigned* p) {
+    if constexpr ((XBFS_STREAM_HINT & BIT) != 0) {
+        unsigned v;
+        asm volatile("ld.global.nc.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(l2_policy_first()));
+        return v;
+    } else {
+        return __ldg(p);
+    }
+}
+template <int BIT>
+__device__ __forceinline__ int ld_ro32(const int* p) {
+    return (int)ld_ro32<BIT>(reinterpret_cast<const unsigned*>(p));
+}
+template <int BIT>
+__device__ __forceinline__ long long ld_ro64(const long long* p) {
+    if constexpr ((XBFS_STREAM_HINT & BIT) != 0) {
+        long long v;
+        asm volatile("ld.global.nc.L2::cache_hint.b64 %0, [%1], %2;" : "=l"(v) : "l"(p), "l"(l2_policy_first()));
+        return v;
+    } else {
+        return *p;
+    }
+}
+
 constexpr int kTile = 2048;          // frontier arcs per td_expand tile
 constexpr int kExpandThreads = 512;  // td_expand block
 constexpr int kBuThreads = 256;      // bu_traverse block (8 warps)
