@@ -909,6 +909,9 @@ __global__ __launch_bounds__(kGenThreads) void k_generate(KArgs a, int role) {
 // kp: where k lives (DevState or the persistent CTA's selector copy); it is
 // re-read for the epilogue instead of keeping k live across the traversal
 // (one register less: the per-level kernel runs at 48 without spills).
+#ifndef XBFS_BU_ALT
+#define XBFS_BU_ALT 1
+#endif
 #if XBFS_BU_PROF
 __device__ unsigned long long g_bu_prof[8];   // profiling build: BU phase cycles of the dense steps
 #endif
@@ -937,6 +940,7 @@ __device__ __forceinline__ void bu_body(const KArgs& a, const int* kp, int* __re
     b.level = level;
     b.parent = parent;
     b.lvl = lvl;
+    b.reverse = XBFS_BU_ALT && (k & 1);   // consecutive BU steps sweep in opposite directions
 #if XBFS_BU_PROF
     b.prof = U * 16 >= a.n ? g_bu_prof : nullptr;   // the dense steps only
 #endif

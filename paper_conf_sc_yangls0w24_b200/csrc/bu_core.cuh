@@ -46,6 +46,7 @@ struct BuView {
     int* level;                       // owned
     int* parent;                      // owned (global ids)
     int lvl;                          // k + 1
+    bool reverse;                     // walk the vertex range downwards (alternating BU steps)
 #if XBFS_BU_PROF
     unsigned long long* prof;         // profiling build: per-phase cycle counters
 #endif
@@ -118,16 +119,21 @@ __device__ __forceinline__ void bu_chunks(const BuView& b, Smem& sm, Publish pub
         const long long ww = cc * kCW + (lane & 7);
         return (cc < nchunks && ww < b.words) ? __ldcg(b.visited + ww) : FULL;
     };
+    // b.reverse: the grid walks the vertex range downwards (every warp its groups in reverse
+    // order), so a BU step that follows another starts where the previous one ended, on the
+    // head32 / level / parent lines still in L2
     const long long st = nw;
-    long long gb = gw;
+    const long long ng = gw < nchunks ? (nchunks - 1 - gw) / (4 * nw) + 1 : 0;   // this warp's groups
+    const long long gstep = b.reverse ? -4 * nw : 4 * nw;
+    long long gb = b.reverse && ng > 0 ? gw + (ng - 1) * 4 * nw : gw;
     unsigned grp_next = load_group(gb, st);
 #if XBFS_BU_PROF
     long long pt[6] = {0, 0, 0, 0, 0, 0};
     long long tq = clock64();
 #endif
-    for (; gb < nchunks; gb += 4 * nw) {
+    for (long long gi = 0; gi < ng; ++gi, gb += gstep) {
         const unsigned grp = grp_next;
-        grp_next = load_group(gb + 4 * nw, nw);
+        grp_next = gi + 1 < ng ? load_group(gb + gstep, nw) : FULL;
         const long long g0 = gb;
         // A sparse group (<= kCW*32 candidates over its 4 chunks, the late BU levels)
         // runs as ONE batch: one first-probe round trip for all of it instead of one

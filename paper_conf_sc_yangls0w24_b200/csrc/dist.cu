@@ -138,6 +138,7 @@ __global__ __launch_bounds__(kBuThreads, 4) void k_bu(DArgs a, int k) {
     b.level = a.level;
     b.parent = a.parent;
     b.lvl = k + 1;
+    b.reverse = false;
 #if XBFS_BU_PROF
     b.prof = nullptr;
 #endif
