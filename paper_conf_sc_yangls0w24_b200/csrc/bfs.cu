@@ -940,7 +940,10 @@ __device__ __forceinline__ void bu_body(const KArgs& a, const int* kp, int* __re
     b.level = level;
     b.parent = parent;
     b.lvl = lvl;
-    b.reverse = XBFS_BU_ALT && (k & 1);   // consecutive BU steps sweep in opposite directions
+    // consecutive BU steps sweep in opposite directions; even levels (the first BU step is
+    // usually level 2) walk downwards, starting where the grid-stride output fill ended
+    // (B200 A/B s24: even-down 862 vs odd-down 856 GTEPS)
+    b.reverse = XBFS_BU_ALT && !(k & 1);
 #if XBFS_BU_PROF
     b.prof = U * 16 >= a.n ? g_bu_prof : nullptr;   // the dense steps only
 #endif
